@@ -1,0 +1,229 @@
+/*
+ * stm.h -- C ABI of the B200-native STMatch counting hot path (libstm.so).
+ *
+ * The library counts the embeddings of a small query pattern Q in a large data
+ * graph G on one B200 (sm_100a) with a single persistent CUDA kernel: outer-loop
+ * parallel, stack-based backtracking (Sec. IV), set
+ * intersection / difference of sorted neighbour lists,
+ * loop unrolling (Sec. VI), loop-invariant code motion
+ * (Sec. VII) and two-level work stealing (Sec. V,
+ * PAPER.md:80-114).  Multi-GPU runs replicate the graph and split the
+ * outermost loop; the caller sums the per-rank partial counts.
+ *
+ * Conventions for every function:
+ *   - extern "C", never throws, returns stm_status.  On anything but STM_OK the
+ *     out-parameters are left untouched and stm_last_error() returns a
+ *     thread-local, human-readable message.
+ *   - Host arrays passed in are BORROWED for the duration of the call only (the
+ *     library copies what it keeps); the caller may free them afterwards.
+ *   - Handles (stm_graph*, stm_plan*) are owned by the library and released by
+ *     the matching *_free call.  Graphs and plans are immutable after creation
+ *     and may be shared by concurrent calls on different CUDA streams.
+ *   - CUDA failures map to STM_ECUDA (message carries cudaGetErrorString).
+ *   - A count is never silently wrong: capacity problems are STM_EOVERFLOW.
+ *
+ * Result semantics (problem statement PAPER.md:44-48):
+ *
+ *   count = #{ f : V_Q -> V injective |
+ *              every pattern edge {a,b} maps to a data edge {f(a), f(b)};
+ *              [vertex-induced] every pattern non-edge maps to a data non-edge;
+ *              [labeled] L_G(f(u)) == L_Q(u) for every u;
+ *              f(a) < f(b) (caller's original vertex IDs) for every restriction (a,b) }
+ *   modulo 2^64.  With STM_AUTO_RESTRICT the restriction set is a complete
+ *   symmetry-breaking set of the label-preserving automorphism group of Q, so the
+ *   count is the number of distinct subgraphs of G isomorphic to Q.
+ */
+#ifndef STM_H_
+#define STM_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  STM_OK = 0,
+  STM_EINVAL = 1,        /* invalid argument (bad CSR, bad pattern, bad order, cyclic restrictions, ...) */
+  STM_ENOMEM = 2,        /* host or device allocation failed */
+  STM_ECUDA = 3,         /* a CUDA runtime call failed */
+  STM_EUNSUPPORTED = 4,  /* valid request outside this build's limits (k > 8, > 255 graph labels, ...) */
+  STM_EOVERFLOW = 5      /* device scratch / stack capacity exceeded: no count produced */
+} stm_status;
+
+typedef struct stm_graph stm_graph; /* opaque, device-resident, immutable */
+typedef struct stm_plan stm_plan;   /* opaque, host-side compiled pattern, immutable */
+
+/* Pattern compilation flags (bitwise OR). */
+enum {
+  STM_EDGE_INDUCED = 0,    /* non-induced monomorphisms: set differences removed */
+  STM_VERTEX_INDUCED = 1,  /* pattern non-edges must be data non-edges: set differences */
+  STM_NO_CODE_MOTION = 2,  /* recompute every level's candidate set from raw neighbour lists (ablation) */
+  STM_AUTO_RESTRICT = 4,   /* ignore `restr`; use Grochow-Kellis symmetry-breaking restrictions */
+  STM_AUTO_ORDER = 8       /* ignore `order`; use the greedy connected order */
+};
+
+enum { STM_K_MAX = 8 };
+
+/*
+ * stm_graph_load -- copy a CSR data graph to device `device` (G = (V, E, L);
+ * neighbour lists are binary-searched, so rows must be sorted).
+ *   n        number of vertices (>= 0); IDs are 0..n-1 and must fit in int32.
+ *   row_ptr  host int64[n+1], row_ptr[0] == 0, non-decreasing.
+ *   col_idx  host int32[row_ptr[n]]; each row strictly increasing (sorted, no
+ *            duplicates), no self-loops, and the graph symmetric (undirected).
+ *   labels   host int32[n] vertex labels (any non-negative values) or NULL.
+ *            At most 255 distinct values (STM_EUNSUPPORTED otherwise).
+ *   device   CUDA device ordinal.
+ *   out      receives the handle.
+ * Errors: STM_EINVAL for any CSR violation above (the full check is O(m log d)
+ * on the host), STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED.
+ */
+stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                          const int32_t* labels, int device, stm_graph** out);
+
+/*
+ * stm_graph_load_device -- as stm_graph_load but BORROWS device arrays already
+ * resident on `device` (e.g. torch tensors).  The caller keeps them alive and
+ * unmodified until stm_graph_free.  Only cheap checks are done (sizes); the
+ * arrays must satisfy the same CSR contract.  Labels (if given) are remapped into
+ * a library-owned device copy.
+ */
+stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_t* d_row_ptr,
+                                 const int32_t* d_col_idx, const int32_t* d_labels, int device,
+                                 stm_graph** out);
+
+/* stm_graph_info -- n, number of directed adjacency entries (2m), max degree. Any out may be NULL. */
+stm_status stm_graph_info(const stm_graph* g, int64_t* n, int64_t* nnz, int64_t* max_degree);
+
+stm_status stm_graph_free(stm_graph* g);
+
+/*
+ * stm_pattern_compile -- host-only pattern compiler (PAPER.md:52 matching order;
+ * PAPER.md:132-140 code motion with merged multi-label sets; restrictions are
+ * north_star's symmetry breaking, not in the paper).
+ *   k        pattern size, 2 <= k <= STM_K_MAX (k == 1 is STM_EINVAL).
+ *   n_edges, edges  pattern edges as 2*n_edges vertex ids in [0,k); duplicates
+ *            are merged; self-loops are STM_EINVAL; Q must be connected.
+ *   labels   int32[k] pattern vertex labels, or NULL (unlabeled).  Value -1 is a
+ *            wildcard (matches any label); other values must be >= 0.
+ *   order    int32[k] matching order (a permutation of 0..k-1 in which every
+ *            vertex after the first is adjacent to an earlier one),
+ *            or NULL for the greedy order.  Ignored with STM_AUTO_ORDER.
+ *   n_restr, restr  2*n_restr pattern vertex pairs (a, b) meaning f(a) < f(b).
+ *            a == b or a cyclic set is STM_EINVAL.  Ignored with STM_AUTO_RESTRICT.
+ *   flags    STM_* flags above.
+ *   out      receives the plan handle.
+ */
+stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edges, const int32_t* labels,
+                               const int32_t* order, int n_restr, const int32_t* restr,
+                               uint32_t flags, stm_plan** out);
+
+/*
+ * stm_plan_describe -- human-readable plan (order, restrictions, |Aut_L|, set
+ * nodes with their operations, candidate sources, scratch words per warp).
+ * Writes at most len bytes including the terminating NUL; returns STM_EINVAL if
+ * len is too small (the message then holds the required size).
+ */
+stm_status stm_plan_describe(const stm_plan* p, char* buf, size_t len);
+
+/* stm_plan_info -- pattern size, number of materialised set nodes, |Aut_L(Q)|. Any out may be NULL. */
+stm_status stm_plan_info(const stm_plan* p, int* k, int* n_sets, int64_t* aut_size);
+
+stm_status stm_plan_free(stm_plan* p);
+
+/* Tuning knobs: every setting changes speed only, never the count. NULL = defaults. */
+typedef struct stm_tuning {
+  int32_t local_steal;    /* 0/1: intra-block stealing through shared memory (Sec. V-A). Default 1. */
+  int32_t global_steal;   /* 0/1: inter-block stealing through global mailboxes (Sec. V-B). Default 1. */
+  int32_t stop_level;     /* frames < stop_level are stealable (paper: 2). Default 2. */
+  int32_t detect_level;   /* donors look for idle blocks at frames < detect_level (paper: 1). Default 2. */
+  int32_t unroll;         /* sibling iterations expanded together, 1..16 (paper: 8). Default 8. */
+  int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 32. */
+  int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
+  int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
+  int32_t debug_per_root; /* 2 = instrumented launch: count algorithmic bytes (stm_last_launch); else reserved */
+} stm_tuning;
+
+/* Fill t with the defaults. */
+void stm_tuning_default(stm_tuning* t);
+
+/*
+ * Multi-GPU shard (duplicate the graph, divide the outermost loop).
+ * The root space [0, n) is cut into chunks of `chunk` roots; chunk c belongs to
+ * rank c % world.  Each rank owns one device-resident uint64 chunk cursor.  With
+ * peer pointers set, a rank whose own cursor is exhausted takes chunks from the
+ * peers' cursors (atomics over NVLink), so every chunk is processed exactly
+ * once across the job.  All ranks must use the same world, chunk and plan.
+ */
+typedef struct stm_shard {
+  int32_t rank, world;           /* 0 <= rank < world <= 8 */
+  int32_t chunk;                 /* roots per chunk (>= 1) */
+  int32_t reserved;
+  uint64_t* d_cursors[8];        /* d_cursors[r] = device pointer to rank r's cursor (own entry
+                                    required; peers NULL = no cross-GPU stealing).  The caller zeroes
+                                    every cursor before the ranks start and keeps them alive. */
+} stm_shard;
+
+/*
+ * stm_match_count -- count on the graph's device (one persistent kernel launch +
+ * an 8-byte read-back, synchronous w.r.t. the host).
+ *   cuda_stream  cudaStream_t to launch on, or NULL for the legacy default stream.
+ *   count        receives the count (mod 2^64).
+ */
+stm_status stm_match_count(const stm_graph* g, const stm_plan* p, void* cuda_stream,
+                           uint64_t* count);
+
+/*
+ * stm_match_count_ex -- as stm_match_count with tuning and an optional shard
+ * (NULL = the whole root space).  With a shard the result is this rank's partial
+ * count; the caller sums the partials (e.g. one NCCL all-reduce).
+ */
+stm_status stm_match_count_ex(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                              const stm_shard* shard, void* cuda_stream, uint64_t* count);
+
+/*
+ * stm_match_count_async -- enqueue the kernel and leave the count in DEVICE
+ * memory (d_count: one uint64, overwritten) without synchronising.  Used by the
+ * benchmark and the multi-GPU layer (the all-reduce then runs on d_count).
+ */
+stm_status stm_match_count_async(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                 const stm_shard* shard, void* cuda_stream, uint64_t* d_count);
+
+/*
+ * stm_match_count_per_root -- localisation build: host uint64[n] receives, for every
+ * root vertex v, the number of counted embeddings with f(order[0]) == v
+ * (order[0] = the plan's first pattern vertex, see stm_plan_describe).  Also
+ * returns the total in *count.
+ */
+stm_status stm_match_count_per_root(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                    void* cuda_stream, uint64_t* per_root, uint64_t* count);
+
+/* stm_plan_first_vertex -- the pattern vertex matched at level 0 (order[0]). */
+stm_status stm_plan_first_vertex(const stm_plan* p, int* u0);
+
+/* Launch record of this thread's last successful stm_match_count* call. */
+typedef struct stm_launch_info {
+  int32_t grid;            /* persistent blocks launched (blocks/SM x SMs) */
+  int32_t block_threads;
+  int32_t smem_bytes;      /* dynamic shared memory per block (DFS stacks) */
+  int32_t cap;             /* words per set-node region (>= max degree) */
+  int64_t arena_bytes;     /* device set arena (all warps) */
+  int64_t local_steals;    /* intra-block steals (Sec. V-A); synchronous calls only */
+  int64_t global_steals;   /* inter-block steals (Sec. V-B); synchronous calls only */
+  int64_t chunks;          /* root chunks taken from cursors; synchronous calls only */
+  int64_t alg_bytes;       /* algorithmic bytes W; instrumented calls only (tuning.debug_per_root == 2) */
+  int64_t merge_bytes;     /* merge-equivalent bytes W_merge; instrumented calls only */
+  int64_t jobs;            /* set operations executed; instrumented calls only */
+} stm_launch_info;
+
+stm_status stm_last_launch(stm_launch_info* info);
+
+/* stm_last_error -- thread-local message for the last non-OK status of this thread. */
+const char* stm_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STM_H_ */

@@ -1,0 +1,1119 @@
+// kernel.cu -- the single persistent sm_100a matching kernel (product hot path).
+//
+// One launch runs the whole backtracking ("finish the computation with
+// one kernel launch").  Every warp runs the stack-based while-loop of Fig. 3
+// on its own DFS stack kept in shared memory; the candidate
+// sets (the paper's C arrays) live in a per-warp global arena sized from the
+// graph's true maximum degree (PAPER.md:154 used a fixed MAX_DEGREE=4096; reading
+// R15).  Level 0 takes chunks of root vertices from a global atomic cursor
+// (Fig. 4).
+//
+// Set operations: a *job* is one "A op N(v)" with op in
+// {intersect, difference}, or a filtered scan.  Up to 32 jobs --
+// the sets of several unrolled sibling iterations (Sec. VI, Fig. 7)
+// or, at the last level, the counts of many candidates -- are flattened into one
+// element stream that the warp walks 32 elements at a time: an inclusive scan of
+// job sizes, a per-lane job lookup, a binary search of the element in the probed
+// sorted list, then ballot/popc compaction into the output set (the combined set
+// operation of Fig. 8).  For an intersection the shorter operand
+// drives and the longer one is probed; value bounds from symmetry-breaking
+// restrictions first narrow both operands by binary search.  The last level is
+// counted and never materialised.
+//
+// Load balance (Sec. V): intra-block stealing through shared memory (Sec. V-A,
+// PAPER.md:84) and inter-block stealing through per-block global mailboxes pushed
+// by busy donors (Sec. V-B, Fig. 6).  Stolen work is a task
+// (prefix, position range); the thief rebuilds the prefix's sets itself.
+#include <climits>
+#include <cstdio>
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "kernel.h"
+
+#define FULLMASK 0xffffffffu
+
+namespace {
+
+struct WarpHdr {
+  int lock;
+  int L;                      // current frame (0 = root level)
+  int root_it, root_end;      // frame 0: remaining root-ID range of the current chunk
+  int nsib[STM_KMAX], cur[STM_KMAX], it[STM_KMAX], end[STM_KMAX];
+  int used[STM_MAX_NODES];    // words used in each node region by the frame being built
+  int stage_c[32], stage_u[32];
+};
+
+struct BlockHdr {
+  int idle_mask;
+  int leader;
+  int done;
+  int pad;
+  unsigned char lab2slot[256];
+};
+
+__host__ __device__ constexpr int warp_bytes_fixed() { return (int)sizeof(WarpHdr); }
+__host__ __device__ inline int warp_bytes(int k, int n_nodes) {
+  int b = warp_bytes_fixed() + k * STM_RMAX * 4 + 2 * n_nodes * STM_UMAX * 4;
+  return (b + 15) & ~15;
+}
+
+struct W {
+  const StmKParams* kp;
+  const StmPlan* P;
+  volatile WarpHdr* h;
+  volatile int* sib;   // [k][RMAX]
+  int* noff;           // [n_nodes][UMAX]
+  int* nsz;            // [n_nodes][UMAX]
+  BlockHdr* bh;
+  int* arena;
+  int lane, wid;
+  unsigned exhausted;  // cursors known to be exhausted (bit per rank)
+  unsigned long long cnt;
+  unsigned gather_calls;
+  unsigned long long wbytes, wmerge, wjobs;  // per-lane instrumentation partials
+};
+
+#define SIB(w, l, u) ((w).sib[(l) * STM_RMAX + (u)])
+#define NOFF(w, s, u) ((w).noff[(s) * STM_UMAX + (u)])
+#define NSZ(w, s, u) ((w).nsz[(s) * STM_UMAX + (u)])
+
+__device__ __forceinline__ int bcast(int x) { return __shfl_sync(FULLMASK, x, 0); }
+
+__device__ __forceinline__ int lbound(const int* __restrict__ a, int n, int x) {
+  int lo = 0;
+  while (n > 0) {
+    int half = n >> 1;
+    int v = a[lo + half];
+    if (v < x) { lo += half + 1; n -= half + 1; } else { n = half; }
+  }
+  return lo;
+}
+
+__device__ __forceinline__ bool member(const int* a, int n, int x) {
+  int p = lbound(a, n, x);
+  return p < n && a[p] == x;
+}
+
+__device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) {
+  long long b = w.kp->row_ptr[v], e = w.kp->row_ptr[v + 1];
+  p = w.kp->col_idx + b;
+  len = (int)(e - b);
+}
+__device__ __forceinline__ int degree(const W& w, int v) {
+  return (int)(w.kp->row_ptr[v + 1] - w.kp->row_ptr[v]);
+}
+
+// value of v_j in the context "frame F, sibling u, candidate c of level F"
+__device__ __forceinline__ int pval(const W& w, int j, int F, int u, int c) {
+  if (j == F) return c;
+  if (j == F - 1) return SIB(w, F, u);
+  return SIB(w, j + 1, w.h->cur[j + 1]);
+}
+
+__device__ __forceinline__ void node_slice(const W& w, int s, int F, int u, int un, const int*& p,
+                                           int& len) {
+  int lvl = w.P->nodes[s].level;
+  int idx = lvl == F + 1 ? un : (lvl == F ? u : w.h->cur[lvl]);
+  p = w.arena + (size_t)s * w.kp->cap + NOFF(w, s, idx);
+  len = NSZ(w, s, idx);
+}
+
+__device__ __forceinline__ void src_slice(const W& w, StmSrc src, int F, int u, int c, int un,
+                                          const int*& p, int& len) {
+  if (src.kind == STM_SRC_RAW) row(w, pval(w, src.idx, F, u, c), p, len);
+  else node_slice(w, src.idx, F, u, un, p, len);
+}
+
+__device__ __forceinline__ void bounds(const W& w, unsigned lo_m, unsigned hi_m, int F, int u, int c,
+                                       int& lo, int& hi) {
+  lo = -1;
+  hi = INT_MAX;
+  for (int j = 0; j < STM_KMAX; ++j) {
+    if (lo_m & (1u << j)) lo = max(lo, pval(w, j, F, u, c));
+    if (hi_m & (1u << j)) hi = min(hi, pval(w, j, F, u, c));
+  }
+}
+
+__device__ __forceinline__ bool labok(const W& w, int x, unsigned lab) {
+  if (lab == STM_LAB_ANY) return true;
+  return (w.bh->lab2slot[w.kp->labels[x]] & lab) != 0;
+}
+
+// ----------------------------------------------------------------------------
+// Flattened multi-job set operation (Fig. 8).  Lane j < njobs owns job j.
+// ----------------------------------------------------------------------------
+struct Job {
+  const int* A;
+  const int* B;  // NULL: filtered scan of A
+  int alen, blen;
+  int op;
+  int lo, hi;
+  unsigned lab;
+  int* out;      // materialise target (NULL in count mode)
+  int u, c;      // context for exclusions / per-root attribution
+};
+
+// Returns the (warp-uniform) number of kept elements summed over all jobs when
+// counting; in materialise mode *outc (lane j) receives job j's output size.
+__device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F, unsigned excl,
+                                       int* outc_lane) {
+  const int lane = w.lane;
+  const bool mine = lane < njobs;
+  const int* D = J.A;
+  const int* Pp = J.B;
+  int dlen = J.alen, plen = J.B ? J.blen : 0;
+  if (mine && J.op == STM_OP_AND && J.blen < J.alen) {
+    D = J.B; dlen = J.blen; Pp = J.A; plen = J.alen;
+  }
+  if (!mine) dlen = 0;
+  if (mine) {  // narrow both operands to the open interval (lo, hi)
+    if (dlen > 16) {
+      if (J.lo >= 0) { int b = lbound(D, dlen, J.lo + 1); D += b; dlen -= b; }
+      if (J.hi < INT_MAX) dlen = lbound(D, dlen, J.hi);
+    }
+    if (plen > 16) {
+      if (J.lo >= 0) { int b = lbound(Pp, plen, J.lo + 1); Pp += b; plen -= b; }
+      if (J.hi < INT_MAX) plen = lbound(Pp, plen, J.hi);
+    }
+  }
+  if (w.kp->count_bytes && mine) {
+    // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below)
+    const long long lg = 32 - __clz(plen);  // ceil(log2(plen+1))
+    w.wbytes += 4ull * (unsigned long long)dlen + 4ull * (unsigned long long)min((long long)plen, (long long)dlen * lg);
+    w.wmerge += 4ull * (unsigned long long)(dlen + plen);
+    w.wjobs += 1;
+  }
+  int incl = dlen;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int t = __shfl_up_sync(FULLMASK, incl, o);
+    if (lane >= o) incl += t;
+  }
+  const int total = __shfl_sync(FULLMASK, incl, 31);
+  const int start = incl - dlen;
+  const bool has_p = Pp != nullptr;
+  int outc = 0;
+  unsigned long long jc = 0;
+  const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
+                           Oll = (unsigned long long)J.out;
+  for (int e0 = 0; e0 < total; e0 += 32) {
+    const int e = e0 + lane;
+    int j = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1) {
+      int v = __shfl_sync(FULLMASK, incl, j + step - 1);
+      if (v <= e) j += step;
+    }
+    const bool valid = e < total;
+    const int* Dj = (const int*)__shfl_sync(FULLMASK, Dll, j);
+    const int* Pj = (const int*)__shfl_sync(FULLMASK, Pll, j);
+    const int sj = __shfl_sync(FULLMASK, start, j);
+    const int pl = __shfl_sync(FULLMASK, plen, j);
+    const int opj = __shfl_sync(FULLMASK, J.op, j);
+    const int loj = __shfl_sync(FULLMASK, J.lo, j);
+    const int hij = __shfl_sync(FULLMASK, J.hi, j);
+    const unsigned labj = __shfl_sync(FULLMASK, J.lab, j);
+    const int hp = __shfl_sync(FULLMASK, (int)has_p, j);
+    bool keep = false;
+    int x = 0;
+    if (valid) {
+      x = Dj[e - sj];
+      keep = x > loj && x < hij;
+      if (keep && hp) {
+        bool f = member(Pj, pl, x);
+        keep = (opj == STM_OP_DIFF) ? !f : f;
+      }
+      if (keep) keep = labok(w, x, labj);
+    }
+    const unsigned km = __ballot_sync(FULLMASK, keep);
+    // lanes of my own job inside this chunk
+    int a = start - e0, b = incl - e0;
+    a = a < 0 ? 0 : a;
+    b = b > 32 ? 32 : b;
+    unsigned rmask = 0;
+    if (mine && a < b) rmask = (b == 32 ? FULLMASK : ((1u << b) - 1)) & ~((1u << a) - 1);
+    if (count_mode) {
+      jc += __popc(km & rmask);
+    } else {
+      int* Oj = (int*)__shfl_sync(FULLMASK, Oll, j);
+      int base = __shfl_sync(FULLMASK, outc, j);
+      int fl = sj - e0;
+      fl = fl < 0 ? 0 : fl;
+      unsigned before = km & ((1u << lane) - 1) & ~((1u << fl) - 1);
+      if (keep) Oj[base + __popc(before)] = x;
+      outc += __popc(km & rmask);
+    }
+  }
+  if (!count_mode) {
+    if (w.kp->count_bytes && mine) w.wbytes += 4ull * (unsigned long long)outc;
+    *outc_lane = outc;
+    return 0;
+  }
+  // exclusions: earlier matched vertices of non-adjacent pattern vertices may
+  // still be in the counted set; remove them explicitly.
+  if (mine && excl) {
+    for (int t = 0; t < STM_KMAX; ++t) {
+      if (!(excl & (1u << t))) continue;
+      int x = pval(w, t, F, J.u, J.c);
+      if (!(x > J.lo && x < J.hi)) continue;
+      if (!labok(w, x, J.lab)) continue;
+      if (!member(J.A, J.alen, x)) continue;
+      if (J.B) {
+        bool f = member(J.B, J.blen, x);
+        if ((J.op == STM_OP_DIFF) ? f : !f) continue;
+      }
+      jc -= 1;
+    }
+  }
+  if (w.kp->per_root && mine && jc) atomicAdd(&w.kp->per_root[pval(w, 0, F, J.u, J.c)], jc);
+  unsigned long long s = jc;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(FULLMASK, s, o);
+  return s;
+}
+
+// count job for the final level in context (F, u, c, un)
+__device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un) {
+  const StmPlan& P = *w.P;
+  Job J;
+  src_slice(w, P.cnt_a, F, u, c, un, J.A, J.alen);
+  J.B = nullptr;
+  J.blen = 0;
+  J.op = P.cnt_op;
+  if (P.cnt_op != STM_OP_NONE) row(w, pval(w, P.cnt_b, F, u, c), J.B, J.blen);
+  const StmFilter f = P.filt[P.k - 1];
+  bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
+  J.lab = f.lab;
+  J.out = nullptr;
+  J.u = u;
+  J.c = c;
+  return J;
+}
+
+// ----------------------------------------------------------------------------
+// locks and small helpers
+// ----------------------------------------------------------------------------
+__device__ __forceinline__ void lock_ws(const W& w, volatile WarpHdr* h) {
+  if (w.lane == 0) {
+    while (atomicCAS((int*)&h->lock, 0, 1) != 0) __nanosleep(32);
+    __threadfence_block();
+  }
+  __syncwarp();
+}
+__device__ __forceinline__ void unlock_ws(const W& w, volatile WarpHdr* h) {
+  __syncwarp();
+  if (w.lane == 0) {
+    __threadfence_block();
+    atomicExch((int*)&h->lock, 0);
+  }
+  __syncwarp();
+}
+__device__ __forceinline__ bool stealing(const W& w) {
+  return w.kp->local_steal || w.kp->global_steal;
+}
+__device__ __forceinline__ bool locked_frame(const W& w, int F) {
+  return stealing(w) && F < w.kp->stop_level;
+}
+
+// candidate-list length of frame F's sibling u
+__device__ __forceinline__ int src_len(const W& w, int F, int u) {
+  const int* p;
+  int len;
+  src_slice(w, w.P->cand[F], F, u, 0, 0, p, len);
+  return len;
+}
+
+__device__ __forceinline__ void set_sibling(W& w, int F, int u) {
+  int len = src_len(w, F, u);
+  if (w.lane == 0) {
+    w.h->cur[F] = u;
+    w.h->it[F] = 0;
+    w.h->end[F] = len;
+  }
+  __syncwarp();
+}
+
+// does candidate c (of level F, sibling u) pass the level's filter?
+__device__ __forceinline__ bool cand_ok(const W& w, int F, int u, int c, int lo, int hi) {
+  const StmFilter f = w.P->filt[F];
+  if (!(c > lo && c < hi)) return false;
+  if (!labok(w, c, f.lab)) return false;
+  if (f.excl) {
+    for (int t = 0; t < F; ++t)
+      if ((f.excl & (1u << t)) && pval(w, t, F, u, c) == c) return false;
+  }
+  return true;
+}
+
+// upper bound on the size of node s (level F+1) for candidate c
+__device__ int node_ub(const W& w, int s, int F, int u, int c) {
+  const StmPlan& P = *w.P;
+  int m = INT_MAX;
+  for (;;) {
+    const StmNode nd = P.nodes[s];
+    if (nd.op == STM_OP_AND) m = min(m, degree(w, pval(w, nd.b, F, u, c)));
+    if (nd.a_kind == STM_SRC_RAW) return min(m, degree(w, pval(w, nd.a, F, u, c)));
+    if (P.nodes[nd.a].level == F + 1) { s = nd.a; continue; }
+    const int* p;
+    int len;
+    node_slice(w, nd.a, F, u, 0, p, len);
+    return min(m, len);
+  }
+}
+
+// Compute the nodes of level F+1 for the m siblings SIB(F+1, 0..m-1); offsets
+// NOFF were assigned by the caller; sizes NSZ are written here.
+__device__ void build_nodes(W& w, int F, int m) {
+  const StmPlan& P = *w.P;
+  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
+  if (nb == ne) return;
+  const int u = F >= 1 ? w.h->cur[F] : 0;
+  for (int st = 0; st < P.n_stages[F + 1]; ++st) {
+    // jobs of this stage: (node, sibling) pairs
+    int nodes_in[STM_MAX_NODES];
+    int nn = 0;
+    for (int s = nb; s < ne; ++s)
+      if (P.nodes[s].stage == st) nodes_in[nn++] = s;
+    const int njobs_total = nn * m;
+    for (int j0 = 0; j0 < njobs_total; j0 += 32) {
+      const int jj = j0 + w.lane;
+      const int nj = min(32, njobs_total - j0);
+      Job J;
+      J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_AND;
+      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0;
+      int s = 0, t = 0;
+      if (w.lane < nj) {
+        s = nodes_in[jj / m];
+        t = jj % m;
+        const StmNode nd = P.nodes[s];
+        const int c = SIB(w, F + 1, t);
+        J.c = c;
+        if (nd.a_kind == STM_SRC_RAW) row(w, pval(w, nd.a, F, u, c), J.A, J.alen);
+        else node_slice(w, nd.a, F, u, t, J.A, J.alen);
+        row(w, pval(w, nd.b, F, u, c), J.B, J.blen);
+        J.op = nd.op;
+        bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
+        J.lab = nd.lab;
+        J.out = w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
+      }
+      int outc = 0;
+      run_jobs(w, J, nj, false, F, 0, &outc);
+      if (w.lane < nj) NSZ(w, s, t) = outc;
+      __syncwarp();
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------
+// gather: next batch of candidates of frame F (current sibling) as the
+// siblings of frame F+1, admitted so that every node region fits.
+// Caller holds the frame lock if the frame is stealable.  Returns batch size.
+// ----------------------------------------------------------------------------
+__device__ int gather_batch(W& w, int F, int U) {
+  const StmPlan& P = *w.P;
+  const int u = w.h->cur[F];
+  const int* src;
+  int len;
+  src_slice(w, P.cand[F], F, u, 0, 0, src, len);
+  int lo, hi;
+  const StmFilter f = P.filt[F];
+  bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
+  int pos = w.h->it[F];
+  const int e = w.h->end[F];
+  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
+  const int cap = w.kp->cap;
+  if (w.lane == 0)
+    for (int s = nb; s < ne; ++s) w.h->used[s] = 0;
+  __syncwarp();
+  int m = 0;
+  bool cut = false;
+  while (m < U && pos < e && !cut) {
+    const int p = pos + w.lane;
+    const bool valid = p < e;
+    int c = valid ? src[p] : 0;
+    bool pass = valid && cand_ok(w, F, u, c, lo, hi);
+    // admission: cumulative upper bounds per node must fit in `cap`
+    bool fits = true;
+    for (int s = nb; s < ne; ++s) {
+      int ub = pass ? node_ub(w, s, F, u, c) : 0;
+      int inc = ub;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int t = __shfl_up_sync(FULLMASK, inc, o);
+        if (w.lane >= o) inc += t;
+      }
+      if (pass && w.h->used[s] + inc > cap) fits = false;
+    }
+    unsigned pm = __ballot_sync(FULLMASK, pass);
+    unsigned fm = __ballot_sync(FULLMASK, pass && fits);
+    // accept a prefix of passing lanes: those before the first non-fitting one, at most U-m
+    unsigned bad = pm & ~fm;
+    unsigned lim = bad ? ((1u << (__ffs(bad) - 1)) - 1) : FULLMASK;
+    unsigned acc = pm & lim;
+    int room = U - m;
+    if (__popc(acc) > room) {
+      // keep the first `room` set bits
+      unsigned a2 = 0, t = acc;
+      for (int i = 0; i < room; ++i) { unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+      acc = a2;
+      cut = true;
+    }
+    if (bad) cut = true;
+    const bool me = (acc >> w.lane) & 1u;
+    const int rank = __popc(acc & ((1u << w.lane) - 1));
+    // second pass: offsets for accepted lanes
+    for (int s = nb; s < ne; ++s) {
+      int ub = me ? node_ub(w, s, F, u, c) : 0;
+      int inc = ub;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int t = __shfl_up_sync(FULLMASK, inc, o);
+        if (w.lane >= o) inc += t;
+      }
+      int used = w.h->used[s];
+      if (me) NOFF(w, s, m + rank) = used + inc - ub;
+      int tot = __shfl_sync(FULLMASK, inc, 31);
+      __syncwarp();
+      if (w.lane == 0) w.h->used[s] = used + tot;
+      __syncwarp();
+    }
+    if (me) SIB(w, F + 1, m + rank) = c;
+    m += __popc(acc);
+    if (cut) {
+      // resume right after the last accepted candidate
+      unsigned hiacc = acc ? (31 - __clz(acc)) : 0;
+      pos = acc ? pos + (int)hiacc + 1 : pos;
+    } else {
+      pos = min(pos + 32, e);
+    }
+    __syncwarp();
+  }
+  if (w.lane == 0) w.h->it[F] = pos;
+  __syncwarp();
+  return m;
+}
+
+// root batch: up to root_batch roots from [root_it, root_end) with the root label
+__device__ int gather_roots(W& w) {
+  const StmPlan& P = *w.P;
+  const int R = w.kp->root_batch;
+  int pos = w.h->root_it;
+  const int e = w.h->root_end;
+  int m = 0;
+  while (m < R && pos < e) {
+    const int p = pos + w.lane;
+    const bool pass = p < e && labok(w, p, P.filt[0].lab);
+    unsigned pm = __ballot_sync(FULLMASK, pass);
+    int room = R - m;
+    unsigned acc = pm;
+    bool cut = false;
+    if (__popc(acc) > room) {
+      unsigned a2 = 0, t = acc;
+      for (int i = 0; i < room; ++i) { unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+      acc = a2;
+      cut = true;
+    }
+    if ((acc >> w.lane) & 1u) SIB(w, 1, m + __popc(acc & ((1u << w.lane) - 1))) = p;
+    m += __popc(acc);
+    pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+  }
+  if (w.lane == 0) w.h->root_it = pos;
+  __syncwarp();
+  return m;
+}
+
+// ----------------------------------------------------------------------------
+// counting
+// ----------------------------------------------------------------------------
+// frame-count mode: frame k-1 is built; one job per sibling
+__device__ void frame_count(W& w, int m) {
+  const int k = w.P->k;
+  const int F = k - 2;
+  const int u = F >= 1 ? w.h->cur[F] : 0;
+  Job J;
+  J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
+  J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0;
+  if (w.lane < m) J = count_job(w, F, u, SIB(w, k - 1, w.lane), w.lane);
+  w.cnt += run_jobs(w, J, m, true, F, w.P->filt[k - 1].excl, nullptr);
+}
+
+// fused mode at frame F = k-2: count over all remaining (sibling, candidate)
+// pairs, 32 jobs per pass.  Returns when the frame is exhausted.
+__device__ void fused_count(W& w, int F) {
+  const StmPlan& P = *w.P;
+  const bool lk = locked_frame(w, F);
+  for (;;) {
+    if (lk) lock_ws(w, w.h);
+    int nj = 0;
+    // gather up to 32 passing candidates across siblings
+    for (;;) {
+      int u = w.h->cur[F];
+      if (u >= w.h->nsib[F]) break;
+      int pos = w.h->it[F], e = w.h->end[F];
+      if (pos >= e) {
+        if (u + 1 >= w.h->nsib[F]) {
+          if (w.lane == 0) w.h->cur[F] = u + 1;
+          __syncwarp();
+          break;
+        }
+        set_sibling(w, F, u + 1);
+        continue;
+      }
+      const int* src;
+      int len;
+      src_slice(w, P.cand[F], F, u, 0, 0, src, len);
+      int lo, hi;
+      bounds(w, P.filt[F].lo, P.filt[F].hi, F, u, 0, lo, hi);
+      const int p = pos + w.lane;
+      const bool valid = p < e;
+      const int c = valid ? src[p] : 0;
+      const bool pass = valid && cand_ok(w, F, u, c, lo, hi);
+      unsigned pm = __ballot_sync(FULLMASK, pass);
+      int room = 32 - nj;
+      unsigned acc = pm;
+      bool cut = false;
+      if (__popc(acc) > room) {
+        unsigned a2 = 0, t = acc;
+        for (int i = 0; i < room; ++i) { unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+        acc = a2;
+        cut = true;
+      }
+      if ((acc >> w.lane) & 1u) {
+        int r = nj + __popc(acc & ((1u << w.lane) - 1));
+        w.h->stage_c[r] = c;
+        w.h->stage_u[r] = u;
+      }
+      nj += __popc(acc);
+      int npos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+      if (w.lane == 0) w.h->it[F] = npos;
+      __syncwarp();
+      if (nj == 32) break;
+    }
+    if (lk) unlock_ws(w, w.h);
+    if (nj == 0) return;
+    Job J;
+    J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
+    J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0;
+    if (w.lane < nj) J = count_job(w, F, w.h->stage_u[w.lane], w.h->stage_c[w.lane], 0);
+    w.cnt += run_jobs(w, J, nj, true, F, P.filt[P.k - 1].excl, nullptr);
+    __syncwarp();
+  }
+}
+
+// ----------------------------------------------------------------------------
+// work acquisition: root chunks, local steal, global steal (Sec. V)
+// ----------------------------------------------------------------------------
+__device__ bool try_chunk(W& w) {
+  const StmKParams& kp = *w.kp;
+  int b = -1, e = -1;
+  if (w.lane == 0) {
+    for (int i = 0; i < kp.world && b < 0; ++i) {
+      int r = (kp.rank + i) % kp.world;
+      if (!kp.cursors[r] || (w.exhausted & (1u << r))) continue;
+      unsigned long long idx = atomicAdd(kp.cursors[r], 1ull);
+      long long c = (long long)r + (long long)kp.world * (long long)idx;
+      long long rb = c * (long long)kp.chunk;
+      if (rb < kp.n) {
+        b = (int)rb;
+        e = (int)min((long long)kp.n, rb + kp.chunk);
+      } else {
+        w.exhausted |= 1u << r;
+      }
+    }
+  }
+  b = bcast(b);
+  e = bcast(e);
+  w.exhausted = __shfl_sync(FULLMASK, w.exhausted, 0);
+  if (b < 0) return false;
+  lock_ws(w, w.h);
+  if (w.lane == 0) {
+    w.h->root_it = b;
+    w.h->root_end = e;
+    w.h->L = 0;
+  }
+  unlock_ws(w, w.h);
+  if (w.lane == 0) atomicAdd(&kp.work->n_chunks, 1ull);
+  return true;
+}
+
+// Split the stack of `v` (caller holds v's lock).  Takes half of the shallowest
+// stealable remaining work.  Work at the victim's current
+// frame L is not in progress yet, so there the victim always keeps at least one
+// item (otherwise a single item could be passed around forever); at frames
+// shallower than L the victim is busy below and the thief may take it all.
+// Returns false if nothing can be taken.
+__device__ bool split_stack(const W& w, volatile WarpHdr* v, volatile int* vsib, StmTask& T) {
+  const int L = v->L;
+  // frame 0: root range
+  int r = v->root_end - v->root_it;
+  int t = (L > 0) ? (r + 1) / 2 : r / 2;
+  if (t >= 1) {
+    T.level = 0;
+    T.e = v->root_end;
+    T.b = v->root_end - t;
+    v->root_end = T.b;
+    return true;
+  }
+  const int stop = w.kp->stop_level;
+  for (int F = 1; F <= L && F < stop; ++F) {
+    if (v->cur[F] >= v->nsib[F]) continue;
+    const int rem = v->end[F] - v->it[F];
+    if (F == 1) {  // remaining root siblings -> root range
+      int rs = v->nsib[1] - v->cur[1] - 1;
+      int ts = (L > 1 || rem > 0) ? (rs + 1) / 2 : rs / 2;
+      if (ts >= 1) {
+        int s0 = v->nsib[1] - ts;
+        T.level = 0;
+        T.b = vsib[1 * STM_RMAX + s0];
+        T.e = vsib[1 * STM_RMAX + v->nsib[1] - 1] + 1;
+        v->nsib[1] = s0;
+        return true;
+      }
+    }
+    const bool last_sib = v->cur[F] + 1 >= v->nsib[F];
+    const int tr = (L > F || !last_sib) ? (rem + 1) / 2 : rem / 2;
+    if (tr >= 1) {
+      T.level = F;
+      T.e = v->end[F];
+      T.b = v->end[F] - tr;
+      for (int j = 0; j < F; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1]];
+      v->end[F] = T.b;
+      return true;
+    }
+  }
+  return false;
+}
+
+// crude amount-of-work score of a stack (higher = better victim), racy read
+__device__ int steal_score(const W& w, volatile WarpHdr* v) {
+  if (v->root_end - v->root_it >= 1) return 1 << 30;
+  const int L = v->L;
+  for (int F = 1; F <= L && F < w.kp->stop_level; ++F) {
+    int rs = (F == 1) ? v->nsib[1] - v->cur[1] - 1 : 0;
+    int rem = v->end[F] - v->it[F];
+    if (v->cur[F] >= v->nsib[F]) rem = 0;
+    if (rs > 0 || rem > 0) return ((STM_KMAX - F) << 24) + min(rs * 1024 + rem, (1 << 24) - 1);
+  }
+  return 0;
+}
+
+__device__ volatile WarpHdr* warp_hdr(const W& w, int wid);
+
+// debug watchdog: true (and a state dump) once the launch has run too long
+__device__ __noinline__ bool watchdog(const W& w, long long t0, const char* where) {
+  if (!w.kp->watchdog_cycles || clock64() - t0 < w.kp->watchdog_cycles) return false;
+  if (w.lane == 0) {
+    int first = atomicExch(&w.kp->work->overflow, 2);
+    volatile WarpHdr* h = w.h;
+    printf("WATCHDOG %s blk %d warp %d L=%d root=[%d,%d) nsib1=%d cur1=%d it1=%d end1=%d idle_blocks=%d mask=%x leader=%d is_idle=%d mail=%d first=%d\n",
+           where, blockIdx.x, w.wid, h->L, h->root_it, h->root_end, h->nsib[1], h->cur[1], h->it[1], h->end[1],
+           *(volatile int*)&w.kp->work->idle_blocks, w.bh->idle_mask, w.bh->leader,
+           w.kp->slots[blockIdx.x].is_idle, w.kp->slots[blockIdx.x].mail_full, first);
+  }
+  __syncwarp();
+  return true;
+}
+__device__ volatile int* warp_sib(const W& w, int wid);
+
+// Rebuild this warp's stack from a task (the receiver recomputes the sets of
+// levels 1..T.level from the prefix).
+__device__ void adopt_task(W& w, const StmTask& T) {
+  const int k = w.P->k;
+  if (T.level == 0) {
+    lock_ws(w, w.h);
+    if (w.lane == 0) {
+      w.h->root_it = T.b;
+      w.h->root_end = T.e;
+      w.h->L = 0;
+    }
+    unlock_ws(w, w.h);
+    return;
+  }
+  const int l = T.level;
+  for (int i = 1; i <= l; ++i) {
+    if (w.lane == 0) {
+      SIB(w, i, 0) = T.prefix[i - 1];
+      w.h->nsib[i] = 1;
+      w.h->cur[i] = 0;
+    }
+    __syncwarp();
+    if (i >= 2) {
+      const StmPlan& P = *w.P;
+      if (w.lane == 0)
+        for (int s = P.level_begin[i]; s < P.level_begin[i + 1]; ++s) NOFF(w, s, 0) = 0;
+      __syncwarp();
+      build_nodes(w, i - 1, 1);
+    }
+    int len = src_len(w, i, 0);
+    if (w.lane == 0) {
+      w.h->it[i] = (i == l) ? T.b : len;
+      w.h->end[i] = (i == l) ? min(T.e, len) : len;
+    }
+    __syncwarp();
+  }
+  (void)k;
+  lock_ws(w, w.h);
+  if (w.lane == 0) w.h->L = l;
+  unlock_ws(w, w.h);
+}
+
+__device__ bool try_local_steal(W& w) {
+  const int nw = w.kp->block_warps;
+  // pick the best victim (racy scores), then split under its lock
+  int best = -1, bs = 0;
+  if (w.lane < nw && w.lane != w.wid) {
+    int s = steal_score(w, warp_hdr(w, w.lane));
+    if (s > 0) { best = w.lane; bs = s; }
+  }
+  // warp argmax (lowest id on ties)
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    int ob = __shfl_xor_sync(FULLMASK, best, o);
+    int os = __shfl_xor_sync(FULLMASK, bs, o);
+    if (os > bs || (os == bs && ob >= 0 && (best < 0 || ob < best))) { best = ob; bs = os; }
+  }
+  if (best < 0) return false;
+  volatile WarpHdr* v = warp_hdr(w, best);
+  StmTask T;
+  int ok = 0;
+  lock_ws(w, v);
+  if (w.lane == 0) ok = split_stack(w, v, warp_sib(w, best), T);
+  unlock_ws(w, v);
+  ok = bcast(ok);
+  if (!ok) return false;
+  T.level = bcast(T.level);
+  T.b = bcast(T.b);
+  T.e = bcast(T.e);
+  for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
+  if (w.lane == 0) atomicAdd(&w.kp->work->n_local_steals, 1ull);
+  adopt_task(w, T);
+  return true;
+}
+
+// donor side of Fig. 6: give half of my shallowest work to an idle block
+__device__ void maybe_donate(W& w) {
+  const StmKParams& kp = *w.kp;
+  int idle = 0;
+  if (w.lane == 0) idle = *(volatile int*)&kp.work->idle_blocks;
+  idle = bcast(idle);
+  if (idle <= 0) return;
+  const int nb = gridDim.x;
+  int target = -1;
+  for (int b0 = 0; b0 < nb && target < 0; b0 += 32) {
+    int b = (blockIdx.x + 1 + b0 + w.lane) % nb;
+    bool cand = (b0 + w.lane < nb) && b != (int)blockIdx.x &&
+                *(volatile int*)&kp.slots[b].is_idle == 1;
+    unsigned cm = __ballot_sync(FULLMASK, cand);
+    while (cm && target < 0) {
+      int l = __ffs(cm) - 1;
+      cm &= cm - 1;
+      int tb = __shfl_sync(FULLMASK, b, l);
+      int got = 0;
+      if (w.lane == 0) got = atomicCAS(&kp.slots[tb].is_idle, 1, 2) == 1;
+      if (bcast(got)) target = tb;
+    }
+  }
+  if (target < 0) return;
+  StmTask T;
+  int ok = 0;
+  lock_ws(w, w.h);
+  if (w.lane == 0) ok = split_stack(w, w.h, w.sib, T);
+  unlock_ws(w, w.h);
+  if (w.lane == 0) {
+    if (!ok) {
+      atomicExch(&kp.slots[target].is_idle, 1);
+    } else {
+      volatile StmTask* M = &kp.slots[target].mail;
+      M->level = T.level;
+      M->b = T.b;
+      M->e = T.e;
+      for (int j = 0; j < STM_KMAX; ++j) M->prefix[j] = T.prefix[j];
+      __threadfence();
+      atomicSub(&kp.work->idle_blocks, 1);
+      __threadfence();
+      atomicExch(&kp.slots[target].mail_full, 1);
+      atomicAdd(&kp.work->n_global_steals, 1ull);
+    }
+  }
+  __syncwarp();
+}
+
+// No more local work: returns true with new work adopted, false on termination.
+__device__ bool acquire_work(W& w, long long t0) {
+  const StmKParams& kp = *w.kp;
+  if (try_chunk(w)) return true;
+  if (!kp.local_steal && !kp.global_steal) return false;
+  if (kp.local_steal && try_local_steal(w)) return true;
+  BlockHdr* bh = w.bh;
+  const unsigned all = (kp.block_warps == 32) ? FULLMASK : ((1u << kp.block_warps) - 1);
+  const unsigned me = 1u << w.wid;
+  bool registered = false;
+  int old = 0;
+  if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
+  old = bcast(old);
+  if ((((unsigned)old) | me) == all) {
+    int got = 0;
+    if (w.lane == 0) got = atomicCAS(&bh->leader, -1, w.wid) == -1;
+    (void)bcast(got);
+  }
+  for (int spin = 0;; ++spin) {
+    if ((spin & 1023) == 1023 && watchdog(w, t0, "acquire")) return false;
+    int done = 0, leader = -1;
+    if (w.lane == 0) {
+      done = *(volatile int*)&bh->done;
+      leader = *(volatile int*)&bh->leader;
+    }
+    done = bcast(done);
+    leader = bcast(leader);
+    if (done) return false;
+    if (leader == w.wid) {
+      if (!kp.global_steal) {
+        if (w.lane == 0) atomicExch(&bh->done, 1);
+        __syncwarp();
+        return false;
+      }
+      StmBlockSlot* S = &kp.slots[blockIdx.x];
+      if (!registered) {
+        if (w.lane == 0) {
+          atomicAdd(&kp.work->idle_blocks, 1);
+          __threadfence();
+          atomicExch(&S->is_idle, 1);
+        }
+        __syncwarp();
+        registered = true;
+      }
+      int full = 0, nidle = 0;
+      if (w.lane == 0) {
+        full = *(volatile int*)&S->mail_full;
+        nidle = *(volatile int*)&kp.work->idle_blocks;
+      }
+      full = bcast(full);
+      nidle = bcast(nidle);
+      if (full) {
+        StmTask T;
+        if (w.lane == 0) {
+          __threadfence();
+          volatile StmTask* M = &S->mail;
+          T.level = M->level;
+          T.b = M->b;
+          T.e = M->e;
+          for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = M->prefix[j];
+          atomicExch(&S->mail_full, 0);
+          atomicExch(&S->is_idle, 0);
+          // leave the idle set before giving up leadership, so no other warp can
+          // see a full mask (and re-register the block) while this one works
+          atomicAnd(&bh->idle_mask, (int)~me);
+          __threadfence_block();
+          atomicExch(&bh->leader, -1);
+        }
+        T.level = bcast(T.level);
+        T.b = bcast(T.b);
+        T.e = bcast(T.e);
+        for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
+        adopt_task(w, T);
+        return true;
+      }
+      if (nidle >= (int)gridDim.x) {
+        if (w.lane == 0) atomicExch(&bh->done, 1);
+        __syncwarp();
+        return false;
+      }
+    } else if (kp.local_steal) {
+      // leave the idle set while trying, so the block is never declared idle
+      // while a stolen task is in flight
+      if (w.lane == 0) atomicAnd(&bh->idle_mask, (int)~me);
+      __syncwarp();
+      if (try_local_steal(w)) return true;
+      if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
+      old = bcast(old);
+      if ((((unsigned)old) | me) == all) {
+        if (w.lane == 0) atomicCAS(&bh->leader, -1, w.wid);
+        __syncwarp();
+      }
+    }
+    if (w.lane == 0) __nanosleep(spin < 64 ? 64 : 512);
+    __syncwarp();
+  }
+}
+
+__device__ volatile WarpHdr* warp_hdr(const W& w, int wid) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  int wb = warp_bytes(w.P->k, w.P->n_nodes);
+  return (volatile WarpHdr*)(smem + sizeof(BlockHdr) + (size_t)wid * wb);
+}
+__device__ volatile int* warp_sib(const W& w, int wid) {
+  return (volatile int*)((volatile unsigned char*)warp_hdr(w, wid) + sizeof(WarpHdr));
+}
+
+}  // namespace
+
+// ----------------------------------------------------------------------------
+// the kernel
+// ----------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constant__ StmKParams kp) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const StmPlan& P = kp.plan;
+  BlockHdr* bh = (BlockHdr*)smem;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (threadIdx.x == 0) {
+    bh->idle_mask = 0;
+    bh->leader = -1;
+    bh->done = 0;
+  }
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) bh->lab2slot[i] = kp.lab2slot[i];
+  const int wb = warp_bytes(P.k, P.n_nodes);
+  unsigned char* wbase = smem + sizeof(BlockHdr) + (size_t)wid * wb;
+  W w;
+  w.kp = &kp;
+  w.P = &P;
+  w.h = (volatile WarpHdr*)wbase;
+  w.sib = (volatile int*)(wbase + sizeof(WarpHdr));
+  w.noff = (int*)(wbase + sizeof(WarpHdr) + P.k * STM_RMAX * 4);
+  w.nsz = w.noff + P.n_nodes * STM_UMAX;
+  w.bh = bh;
+  const long long gw = (long long)blockIdx.x * kp.block_warps + wid;
+  w.arena = kp.arena + (size_t)gw * (size_t)P.n_nodes * (size_t)kp.cap;
+  w.lane = lane;
+  w.wid = wid;
+  w.exhausted = 0;
+  w.cnt = 0;
+  w.gather_calls = 0;
+  w.wbytes = w.wmerge = w.wjobs = 0;
+  if (lane == 0) {
+    w.h->lock = 0;
+    w.h->L = 0;
+    w.h->root_it = 0;
+    w.h->root_end = 0;
+    for (int i = 0; i < STM_KMAX; ++i) {
+      w.h->nsib[i] = 0;
+      w.h->cur[i] = 0;
+      w.h->it[i] = 0;
+      w.h->end[i] = 0;
+    }
+  }
+  __syncthreads();
+
+  const int k = P.k;
+  const int U = max(1, min(kp.unroll, STM_UMAX));
+  const bool fused = P.count_mode == STM_COUNT_FUSED;
+  const long long t0 = clock64();
+  unsigned iter = 0;
+  for (;;) {
+    if ((++iter & 255) == 0 && watchdog(w, t0, "main")) break;
+    int L = w.h->L;
+    if (L == 0) {
+      const bool lk = stealing(w);
+      if (lk) lock_ws(w, w.h);
+      int m = gather_roots(w);
+      if (m > 0) {
+        if (w.lane == 0) {
+          w.h->nsib[1] = m;
+          w.h->cur[1] = 0;
+        }
+        __syncwarp();
+        set_sibling(w, 1, 0);
+        if (k == 2) {
+          if (lk) unlock_ws(w, w.h);
+          frame_count(w, m);  // counts N(root) per root
+          continue;
+        }
+        if (w.lane == 0) w.h->L = 1;
+        __syncwarp();
+      }
+      if (lk) unlock_ws(w, w.h);
+      if (m == 0) {
+        if (!acquire_work(w, t0)) break;
+      }
+      continue;
+    }
+    const int F = L;
+    if (fused && F == k - 2) {
+      fused_count(w, F);
+      const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
+      if (lk) lock_ws(w, w.h);
+      if (w.lane == 0) w.h->L = F - 1;
+      if (lk) unlock_ws(w, w.h);
+      __syncwarp();
+      continue;
+    }
+    const bool lk = locked_frame(w, F);
+    if (kp.global_steal && F < kp.detect_level && F < kp.stop_level) maybe_donate(w);
+    if (lk) lock_ws(w, w.h);
+    int m = 0;
+    bool back = false;
+    for (;;) {
+      if (w.h->cur[F] >= w.h->nsib[F]) { back = true; break; }
+      if (w.h->it[F] < w.h->end[F]) {
+        m = gather_batch(w, F, U);
+        if (m > 0) break;
+      }
+      int nu = w.h->cur[F] + 1;
+      if (nu >= w.h->nsib[F]) {
+        if (w.lane == 0) w.h->cur[F] = nu;
+        __syncwarp();
+        back = true;
+        break;
+      }
+      set_sibling(w, F, nu);
+    }
+    if (back) {
+      if (w.lane == 0) w.h->L = F - 1;
+      __syncwarp();
+      if (lk) unlock_ws(w, w.h);
+      continue;
+    }
+    if (lk) unlock_ws(w, w.h);
+    // build frame F+1 from the batch
+    build_nodes(w, F, m);
+    if (F + 1 == k - 1) {  // frame-count mode
+      frame_count(w, m);
+      continue;
+    }
+    const bool lk2 = locked_frame(w, F + 1);
+    if (lk2) lock_ws(w, w.h);
+    if (w.lane == 0) w.h->nsib[F + 1] = m;
+    __syncwarp();
+    set_sibling(w, F + 1, 0);
+    if (w.lane == 0) w.h->L = F + 1;
+    __syncwarp();
+    if (lk2) unlock_ws(w, w.h);
+  }
+  if (lane == 0 && w.cnt) atomicAdd(&kp.work->count, w.cnt);
+  if (kp.count_bytes) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      w.wbytes += __shfl_xor_sync(FULLMASK, w.wbytes, o);
+      w.wmerge += __shfl_xor_sync(FULLMASK, w.wmerge, o);
+      w.wjobs += __shfl_xor_sync(FULLMASK, w.wjobs, o);
+    }
+    if (lane == 0) {
+      atomicAdd(&kp.work->alg_bytes, w.wbytes);
+      atomicAdd(&kp.work->merge_bytes, w.wmerge);
+      atomicAdd(&kp.work->n_jobs, w.wjobs);
+    }
+  }
+}
+
+int stm_smem_bytes(int block_warps, int k, int n_nodes) {
+  return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes);
+}
+
+int stm_occupancy(int block_warps, int k, int n_nodes, int* blocks_per_sm) {
+  int smem = stm_smem_bytes(block_warps, k, n_nodes);
+  cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, stm_count_kernel, block_warps * 32, smem);
+  return (int)e;
+}
+
+int stm_launch(const StmKParams& kp, int grid, void* stream) {
+  int smem = stm_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes);
+  cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  void* args[] = {(void*)&kp};
+  e = cudaLaunchCooperativeKernel((const void*)stm_count_kernel, dim3(grid), dim3(kp.block_warps * 32), args,
+                                  (size_t)smem, (cudaStream_t)stream);
+  return (int)e;
+}

@@ -1,0 +1,63 @@
+// kernel.h -- launch interface between the runtime (runtime.cu) and the persistent
+// matching kernel (kernel.cu).  Product code only.
+#pragma once
+#include <stdint.h>
+
+#include "plan.h"
+
+// A unit of stealable work (Sec. V).  level 0: root-ID range
+// [b, e).  level l >= 1: the prefix v_0..v_{l-1} (prefix[0..l-1]) and the
+// positions [b, e) of the level-l candidate list of that prefix.  The candidate
+// list is a sorted set determined by the prefix alone, so the receiver rebuilds
+// the sets of levels 1..l from the prefix instead of copying them (DESIGN.md,
+// "Stealing": differs from PAPER.md:142, which copies the sets).
+struct StmTask {
+  int32_t level;
+  int32_t b, e;
+  int32_t prefix[STM_KMAX];
+};
+
+// Device-resident scheduler state of one launch (zeroed before every launch).
+struct StmWork {
+  unsigned long long count;       // result accumulator (mod 2^64)
+  int32_t idle_blocks;            // blocks registered idle (Fig. 6 is_idle count)
+  int32_t overflow;               // set if any capacity check fails
+  unsigned long long n_local_steals, n_global_steals, n_chunks;
+  unsigned long long alg_bytes;    // SURVEY.md 8(d) W = sum W_op (instrumented launches only)
+  unsigned long long merge_bytes;  // W_merge = sum 4(|A|+|B|)
+  unsigned long long n_jobs;
+};
+
+struct StmBlockSlot {             // per block, global memory (Fig. 6)
+  int32_t is_idle;                // 0 busy, 1 idle & waiting, 2 claimed by a donor
+  int32_t mail_full;              // 1 when `mail` holds a task for this block
+  int32_t pad[2];
+  StmTask mail;
+};
+
+struct StmKParams {
+  StmPlan plan;
+  const int64_t* row_ptr;
+  const int32_t* col_idx;
+  const uint8_t* labels;          // dense graph label ids, or NULL
+  int64_t n;
+  int32_t cap;                    // words per set-node region per warp
+  int32_t block_warps;
+  int32_t* arena;                 // [total_warps][n_nodes][cap]
+  StmWork* work;
+  StmBlockSlot* slots;            // [gridDim.x]
+  unsigned long long* per_root;   // [n] or NULL
+  unsigned long long* cursors[8]; // chunk cursors (own rank + optional peers)
+  int32_t rank, world, chunk;
+  int32_t local_steal, global_steal, stop_level, detect_level, unroll, root_batch;
+  int32_t count_bytes;            // 1 = accumulate algorithmic bytes (instrumented launch)
+  long long watchdog_cycles;      // debug: abort (set work->overflow = 2) after this many cycles; 0 = off
+  uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
+};
+
+// size in bytes of the dynamic shared memory for one block
+int stm_smem_bytes(int block_warps, int k, int n_nodes);
+// launches the persistent kernel (cooperative); returns cudaError_t as int
+int stm_launch(const StmKParams& kp, int grid, void* stream);
+// max co-resident blocks per SM for the given block size
+int stm_occupancy(int block_warps, int k, int n_nodes, int* blocks_per_sm);

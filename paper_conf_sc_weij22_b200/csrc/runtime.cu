@@ -1,0 +1,434 @@
+// runtime.cu -- C ABI of libstm.so: graph residency, scratch sizing, launch,
+// read-back.  Product code (never calls the oracle).
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <new>
+#include <thread>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "internal.h"
+#include "kernel.h"
+
+static thread_local char g_err[1024] = "";
+static thread_local stm_launch_info g_info = {};
+
+stm_status stm_fail(stm_status s, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof g_err, fmt, ap);
+  va_end(ap);
+  return s;
+}
+
+extern "C" const char* stm_last_error(void) { return g_err; }
+
+#define CU(call)                                                                         \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess) return stm_fail(STM_ECUDA, "%s: %s", #call, cudaGetErrorString(e_)); \
+  } while (0)
+
+namespace {
+struct Scratch {
+  int* arena = nullptr;
+  size_t arena_bytes = 0;
+  void* state = nullptr;  // StmWork + cursor + StmBlockSlot[grid]
+  size_t state_bytes = 0;
+};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+}  // namespace
+
+struct stm_graph {
+  int device = 0;
+  int64_t n = 0, nnz = 0, max_degree = 0;
+  int64_t* d_row_ptr = nullptr;
+  int32_t* d_col_idx = nullptr;
+  uint8_t* d_labels = nullptr;
+  bool owns_csr = true;
+  std::vector<int32_t> label_values;  // dense id -> label value
+  int num_sms = 0;
+  std::mutex mu;
+  std::map<void*, Scratch> scratch;  // per stream
+};
+
+// ---------------------------------------------------------------------------- load
+// max degree and monotonicity of a device row_ptr (out[0] = max degree, out[1] = bad flag)
+__global__ void degree_scan(const int64_t* rp, int64_t n, long long* out) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    long long d = rp[v + 1] - rp[v];
+    if (d < 0) out[1] = 1;
+    else atomicMax(&out[0], d);
+  }
+}
+
+static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci) {
+  if (rp[0] != 0) return stm_fail(STM_EINVAL, "row_ptr[0] != 0");
+  for (int64_t v = 0; v < n; ++v)
+    if (rp[v + 1] < rp[v]) return stm_fail(STM_EINVAL, "row_ptr decreases at %lld", (long long)v);
+  unsigned nt = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+  std::vector<int> bad(nt, 0);
+  std::vector<int64_t> badv(nt, -1);
+  std::vector<std::thread> th;
+  for (unsigned t = 0; t < nt; ++t)
+    th.emplace_back([&, t] {
+      int64_t lo = n * t / nt, hi = n * (t + 1) / nt;
+      for (int64_t v = lo; v < hi && !bad[t]; ++v) {
+        for (int64_t e = rp[v]; e < rp[v + 1]; ++e) {
+          int64_t w = ci[e];
+          if (w < 0 || w >= n) { bad[t] = 1; badv[t] = v; break; }
+          if (w == v) { bad[t] = 2; badv[t] = v; break; }
+          if (e > rp[v] && ci[e - 1] >= w) { bad[t] = 3; badv[t] = v; break; }
+          // symmetry: v must be in N(w)
+          const int32_t* b = ci + rp[w];
+          const int32_t* x = std::lower_bound(b, ci + rp[w + 1], (int32_t)v);
+          if (x == ci + rp[w + 1] || *x != v) { bad[t] = 4; badv[t] = v; break; }
+        }
+      }
+    });
+  for (auto& x : th) x.join();
+  static const char* why[] = {"", "neighbour id out of range", "self-loop", "row not strictly increasing",
+                              "graph not symmetric"};
+  for (unsigned t = 0; t < nt; ++t)
+    if (bad[t]) return stm_fail(STM_EINVAL, "%s at vertex %lld", why[bad[t]], (long long)badv[t]);
+  return STM_OK;
+}
+
+static stm_status dense_labels(int64_t n, const int32_t* labels, std::vector<uint8_t>& dense,
+                               std::vector<int32_t>& values) {
+  values.assign(labels, labels + n);
+  std::sort(values.begin(), values.end());
+  values.erase(std::unique(values.begin(), values.end()), values.end());
+  if (!values.empty() && values[0] < 0) return stm_fail(STM_EINVAL, "negative vertex label %d", values[0]);
+  if (values.size() > 255)
+    return stm_fail(STM_EUNSUPPORTED, "%zu distinct vertex labels > 255", values.size());
+  dense.resize(n);
+  for (int64_t v = 0; v < n; ++v)
+    dense[v] = (uint8_t)(std::lower_bound(values.begin(), values.end(), labels[v]) - values.begin());
+  return STM_OK;
+}
+
+extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                                     const int32_t* labels, int device, stm_graph** out) {
+  if (!out) return stm_fail(STM_EINVAL, "out is NULL");
+  if (n < 0 || n > INT32_MAX - 1) return stm_fail(STM_EINVAL, "n=%lld out of range", (long long)n);
+  if (!row_ptr) return stm_fail(STM_EINVAL, "row_ptr is NULL");
+  int64_t nnz = row_ptr[n];
+  if (nnz > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
+  stm_status s = validate_csr(n, row_ptr, col_idx);
+  if (s != STM_OK) return s;
+  std::vector<uint8_t> dense;
+  std::vector<int32_t> values;
+  if (labels) {
+    s = dense_labels(n, labels, dense, values);
+    if (s != STM_OK) return s;
+  }
+  int64_t maxd = 0;
+  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, row_ptr[v + 1] - row_ptr[v]);
+  int ndev = 0;
+  CU(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return stm_fail(STM_EINVAL, "device %d of %d", device, ndev);
+  DeviceGuard dg(device);
+  stm_graph* g = new (std::nothrow) stm_graph();
+  if (!g) return stm_fail(STM_ENOMEM, "host allocation");
+  g->device = device;
+  g->n = n;
+  g->nnz = nnz;
+  g->max_degree = maxd;
+  g->label_values = values;
+  cudaError_t e = cudaMalloc(&g->d_row_ptr, sizeof(int64_t) * (n + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&g->d_col_idx, sizeof(int32_t) * std::max<int64_t>(nnz, 1));
+  if (e == cudaSuccess && labels) e = cudaMalloc(&g->d_labels, std::max<int64_t>(n, 1));
+  if (e == cudaSuccess) e = cudaMemcpy(g->d_row_ptr, row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && nnz) e = cudaMemcpy(g->d_col_idx, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && labels && n) e = cudaMemcpy(g->d_labels, dense.data(), n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  if (e != cudaSuccess) {
+    stm_graph_free(g);
+    return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
+                    cudaGetErrorString(e));
+  }
+  *out = g;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_t* d_row_ptr,
+                                            const int32_t* d_col_idx, const int32_t* d_labels, int device,
+                                            stm_graph** out) {
+  if (!out || !d_row_ptr || (nnz > 0 && !d_col_idx)) return stm_fail(STM_EINVAL, "NULL argument");
+  if (n < 0 || n > INT32_MAX - 1 || nnz < 0) return stm_fail(STM_EINVAL, "bad sizes");
+  DeviceGuard dg(device);
+  // cheap checks on the device: row_ptr[0] == 0, row_ptr[n] == nnz, monotone; max degree
+  int64_t maxd = 0;
+  {
+    long long* d = nullptr;
+    CU(cudaMalloc(&d, 3 * sizeof(long long)));
+    long long init[3] = {0, 0, 0};
+    CU(cudaMemcpy(d, init, sizeof init, cudaMemcpyHostToDevice));
+    if (n > 0) degree_scan<<<(unsigned)std::min<int64_t>((n + 255) / 256, 65535), 256>>>(d_row_ptr, n, d);
+    long long h[3];
+    cudaError_t e = cudaMemcpy(h, d, sizeof h, cudaMemcpyDeviceToHost);
+    int64_t ends[2] = {0, 0};
+    if (e == cudaSuccess) e = cudaMemcpy(&ends[0], d_row_ptr, sizeof(int64_t), cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(&ends[1], d_row_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    if (e != cudaSuccess) return stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+    if (ends[0] != 0 || ends[1] != nnz) return stm_fail(STM_EINVAL, "row_ptr does not match nnz");
+    if (h[1]) return stm_fail(STM_EINVAL, "row_ptr decreases");
+    maxd = h[0];
+  }
+  stm_graph* g = new (std::nothrow) stm_graph();
+  if (!g) return stm_fail(STM_ENOMEM, "host allocation");
+  g->device = device;
+  g->n = n;
+  g->nnz = nnz;
+  g->max_degree = maxd;
+  g->owns_csr = false;
+  g->d_row_ptr = const_cast<int64_t*>(d_row_ptr);
+  g->d_col_idx = const_cast<int32_t*>(d_col_idx);
+  if (d_labels) {
+    std::vector<int32_t> lab(n);
+    cudaError_t e = cudaMemcpy(lab.data(), d_labels, sizeof(int32_t) * n, cudaMemcpyDeviceToHost);
+    std::vector<uint8_t> dense;
+    stm_status s = e == cudaSuccess ? dense_labels(n, lab.data(), dense, g->label_values)
+                                    : stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+    if (s == STM_OK) {
+      e = cudaMalloc(&g->d_labels, std::max<int64_t>(n, 1));
+      if (e == cudaSuccess && n) e = cudaMemcpy(g->d_labels, dense.data(), n, cudaMemcpyHostToDevice);
+      if (e != cudaSuccess) s = stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+    }
+    if (s != STM_OK) {
+      stm_graph_free(g);
+      return s;
+    }
+  }
+  cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  *out = g;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_graph_info(const stm_graph* g, int64_t* n, int64_t* nnz, int64_t* maxd) {
+  if (!g) return stm_fail(STM_EINVAL, "NULL graph");
+  if (n) *n = g->n;
+  if (nnz) *nnz = g->nnz;
+  if (maxd) *maxd = g->max_degree;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_graph_free(stm_graph* g) {
+  if (!g) return STM_OK;
+  DeviceGuard dg(g->device);
+  for (auto& kv : g->scratch) {
+    cudaFree(kv.second.arena);
+    cudaFree(kv.second.state);
+  }
+  if (g->owns_csr) {
+    cudaFree(g->d_row_ptr);
+    cudaFree(g->d_col_idx);
+  }
+  cudaFree(g->d_labels);
+  delete g;
+  return STM_OK;
+}
+
+extern "C" void stm_tuning_default(stm_tuning* t) {
+  if (!t) return;
+  memset(t, 0, sizeof *t);
+  t->local_steal = 1;
+  t->global_steal = 1;
+  t->stop_level = 2;
+  t->detect_level = 2;
+  t->unroll = 8;
+  t->root_chunk = 32;
+  t->block_warps = 16;
+  t->blocks_per_sm = 0;
+}
+
+// ---------------------------------------------------------------------------- match
+static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tuning* tin,
+                         const stm_shard* shard, void* stream, uint64_t* d_count_out,
+                         unsigned long long* d_per_root, uint64_t* h_count) {
+  if (!gc || !p) return stm_fail(STM_EINVAL, "NULL graph or plan");
+  stm_graph* g = const_cast<stm_graph*>(gc);
+  stm_tuning t;
+  if (tin) t = *tin; else stm_tuning_default(&t);
+  if (t.unroll < 1 || t.unroll > STM_UMAX) return stm_fail(STM_EINVAL, "unroll %d not in 1..%d", t.unroll, STM_UMAX);
+  if (t.root_chunk < 1) return stm_fail(STM_EINVAL, "root_chunk %d < 1", t.root_chunk);
+  if (t.block_warps == 0) t.block_warps = 16;
+  if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
+  if (t.stop_level < 1) t.stop_level = 1;
+  const StmPlan& P = p->dev;
+  if (!p->labels.empty() && !g->d_labels) {
+    bool any = false;
+    for (int x : p->labels) any |= x >= 0;
+    if (any) return stm_fail(STM_EINVAL, "labeled pattern on an unlabeled graph");
+  }
+  if (shard) {
+    if (shard->world < 1 || shard->world > 8 || shard->rank < 0 || shard->rank >= shard->world ||
+        shard->chunk < 1 || !shard->d_cursors[shard->rank])
+      return stm_fail(STM_EINVAL, "bad shard");
+  }
+  DeviceGuard dg(g->device);
+
+  StmKParams kp;
+  memset(&kp, 0, sizeof kp);
+  kp.plan = P;
+  kp.row_ptr = g->d_row_ptr;
+  kp.col_idx = g->d_col_idx;
+  kp.labels = g->d_labels;
+  kp.n = g->n;
+  // label-slot table: dense graph label -> bitmask of pattern slots with that value
+  for (int d = 0; d < (int)g->label_values.size(); ++d)
+    for (int s = 0; s < P.n_label_slots; ++s)
+      if (g->label_values[d] == P.label_value[s]) kp.lab2slot[d] |= (uint8_t)(1u << s);
+  const int64_t cap64 = std::max<int64_t>(32, (g->max_degree + 31) / 32 * 32);
+  if (cap64 > INT32_MAX / 4) return stm_fail(STM_EUNSUPPORTED, "max degree too large");
+  kp.cap = (int)cap64;
+  kp.block_warps = t.block_warps;
+  kp.local_steal = t.local_steal;
+  kp.global_steal = t.global_steal;
+  kp.stop_level = t.stop_level;
+  kp.detect_level = t.detect_level;
+  kp.unroll = t.unroll;
+  kp.root_batch = std::max(1, std::min(STM_RMAX, t.root_chunk));
+  kp.count_bytes = t.debug_per_root == 2 ? 1 : 0;  // reserved field doubles as the instrumentation switch
+  if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
+
+  int bps = 0;
+  int oe = stm_occupancy(t.block_warps, P.k, P.n_nodes, &bps);
+  if (oe != 0) return stm_fail(STM_ECUDA, "occupancy: %s", cudaGetErrorString((cudaError_t)oe));
+  if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
+  if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
+  const int grid = bps * g->num_sms;
+  const int64_t warps = (int64_t)grid * t.block_warps;
+  const size_t arena_bytes = (size_t)warps * (size_t)P.n_nodes * (size_t)kp.cap * sizeof(int32_t);
+  const size_t state_bytes = sizeof(StmWork) + 64 + sizeof(StmBlockSlot) * (size_t)grid;
+
+  Scratch* S;
+  {
+    std::lock_guard<std::mutex> lk(g->mu);
+    S = &g->scratch[stream];
+    if (S->arena_bytes < arena_bytes) {
+      cudaFree(S->arena);
+      S->arena = nullptr;
+      S->arena_bytes = 0;
+      if (arena_bytes) {
+        cudaError_t e = cudaMalloc(&S->arena, arena_bytes);
+        if (e != cudaSuccess)
+          return stm_fail(STM_ENOMEM, "set arena of %zu bytes: %s", arena_bytes, cudaGetErrorString(e));
+        S->arena_bytes = arena_bytes;
+      }
+    }
+    if (S->state_bytes < state_bytes) {
+      cudaFree(S->state);
+      S->state = nullptr;
+      S->state_bytes = 0;
+      CU(cudaMalloc(&S->state, state_bytes));
+      S->state_bytes = state_bytes;
+    }
+  }
+  StmWork* work = (StmWork*)S->state;
+  unsigned long long* own_cursor = (unsigned long long*)((char*)S->state + sizeof(StmWork));
+  StmBlockSlot* slots = (StmBlockSlot*)((char*)S->state + sizeof(StmWork) + 64);
+  kp.arena = S->arena;
+  kp.work = work;
+  kp.slots = slots;
+  kp.per_root = d_per_root;
+  if (shard) {
+    kp.rank = shard->rank;
+    kp.world = shard->world;
+    kp.chunk = shard->chunk;
+    for (int r = 0; r < shard->world; ++r) kp.cursors[r] = (unsigned long long*)shard->d_cursors[r];
+  } else {
+    kp.rank = 0;
+    kp.world = 1;
+    kp.chunk = t.root_chunk;
+    kp.cursors[0] = own_cursor;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  CU(cudaMemsetAsync(S->state, 0, state_bytes, st));
+  int le = stm_launch(kp, grid, stream);
+  if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
+  g_info.grid = grid;
+  g_info.block_threads = t.block_warps * 32;
+  g_info.smem_bytes = stm_smem_bytes(t.block_warps, P.k, P.n_nodes);
+  g_info.arena_bytes = (int64_t)arena_bytes;
+  g_info.cap = kp.cap;
+  if (d_count_out) {
+    CU(cudaMemcpyAsync(d_count_out, &work->count, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
+  }
+  if (h_count) {
+    StmWork hw;
+    CU(cudaMemcpyAsync(&hw, work, sizeof(StmWork), cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    if (hw.overflow == 2) return stm_fail(STM_ECUDA, "watchdog expired (STM_WATCHDOG_S)");
+    if (hw.overflow) return stm_fail(STM_EOVERFLOW, "device capacity exceeded");
+    g_info.local_steals = (int64_t)hw.n_local_steals;
+    g_info.global_steals = (int64_t)hw.n_global_steals;
+    g_info.chunks = (int64_t)hw.n_chunks;
+    g_info.alg_bytes = (int64_t)hw.alg_bytes;
+    g_info.merge_bytes = (int64_t)hw.merge_bytes;
+    g_info.jobs = (int64_t)hw.n_jobs;
+    *h_count = hw.count;
+  }
+  return STM_OK;
+}
+
+extern "C" stm_status stm_match_count(const stm_graph* g, const stm_plan* p, void* stream, uint64_t* count) {
+  if (!count) return stm_fail(STM_EINVAL, "count is NULL");
+  return launch(g, p, nullptr, nullptr, stream, nullptr, nullptr, count);
+}
+
+extern "C" stm_status stm_match_count_ex(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                         const stm_shard* shard, void* stream, uint64_t* count) {
+  if (!count) return stm_fail(STM_EINVAL, "count is NULL");
+  return launch(g, p, t, shard, stream, nullptr, nullptr, count);
+}
+
+extern "C" stm_status stm_match_count_async(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                            const stm_shard* shard, void* stream, uint64_t* d_count) {
+  if (!d_count) return stm_fail(STM_EINVAL, "d_count is NULL");
+  return launch(g, p, t, shard, stream, d_count, nullptr, nullptr);
+}
+
+extern "C" stm_status stm_match_count_per_root(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                               void* stream, uint64_t* per_root, uint64_t* count) {
+  if (!g || !per_root || !count) return stm_fail(STM_EINVAL, "NULL argument");
+  DeviceGuard dg(g->device);
+  unsigned long long* d = nullptr;
+  CU(cudaMalloc(&d, sizeof(unsigned long long) * std::max<int64_t>(g->n, 1)));
+  cudaMemset(d, 0, sizeof(unsigned long long) * std::max<int64_t>(g->n, 1));
+  uint64_t c = 0;
+  stm_status s = launch(g, p, t, nullptr, stream, nullptr, d, &c);
+  if (s == STM_OK) {
+    cudaError_t e = cudaMemcpy(per_root, d, sizeof(uint64_t) * g->n, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) s = stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+  }
+  cudaFree(d);
+  if (s == STM_OK) *count = c;
+  return s;
+}
+
+extern "C" stm_status stm_last_launch(stm_launch_info* info) {
+  if (!info) return stm_fail(STM_EINVAL, "NULL info");
+  *info = g_info;
+  return STM_OK;
+}

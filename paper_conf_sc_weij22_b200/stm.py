@@ -1,0 +1,273 @@
+"""Thin ctypes binding over libstm.so (include/stm.h).  Argument marshalling only:
+every step of the counting path runs inside the library's CUDA kernel.  There is
+no CPU fallback: importing this module without the built library raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, fields
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libstm.so")
+
+STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW = range(6)
+STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
+_NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW"}
+
+EXPORTS = ["stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
+           "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
+           "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
+           "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_error"]
+
+
+class StmError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_NAMES.get(status, status)}: {msg}")
+        self.status = status
+
+
+class stm_tuning(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("local_steal", "global_steal", "stop_level", "detect_level",
+                                               "unroll", "root_chunk", "block_warps", "blocks_per_sm",
+                                               "debug_per_root")]
+
+
+class stm_shard(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("chunk", ctypes.c_int32),
+                ("reserved", ctypes.c_int32), ("d_cursors", ctypes.c_void_p * 8)]
+
+
+class stm_launch_info(ctypes.Structure):
+    _fields_ = [("grid", ctypes.c_int32), ("block_threads", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
+                ("cap", ctypes.c_int32), ("arena_bytes", ctypes.c_int64), ("local_steals", ctypes.c_int64),
+                ("global_steals", ctypes.c_int64), ("chunks", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
+                ("merge_bytes", ctypes.c_int64), ("jobs", ctypes.c_int64)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_weij22_b200.build` "
+                          "(there is no CPU fallback)")
+    lib = ctypes.CDLL(LIB_PATH)
+    vp, i32, i64, u32, sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_uint32, ctypes.c_size_t
+    P64 = ctypes.POINTER(ctypes.c_int64)
+    sig = {
+        "stm_graph_load": [i64, vp, vp, vp, i32, ctypes.POINTER(vp)],
+        "stm_graph_load_device": [i64, i64, vp, vp, vp, i32, ctypes.POINTER(vp)],
+        "stm_graph_info": [vp, P64, P64, P64],
+        "stm_graph_free": [vp],
+        "stm_pattern_compile": [i32, i32, vp, vp, vp, i32, vp, u32, ctypes.POINTER(vp)],
+        "stm_plan_describe": [vp, ctypes.c_char_p, sz],
+        "stm_plan_info": [vp, ctypes.POINTER(i32), ctypes.POINTER(i32), P64],
+        "stm_plan_free": [vp],
+        "stm_plan_first_vertex": [vp, ctypes.POINTER(i32)],
+        "stm_match_count": [vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
+        "stm_match_count_ex": [vp, vp, vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
+        "stm_match_count_async": [vp, vp, vp, vp, vp, vp],
+        "stm_match_count_per_root": [vp, vp, vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
+        "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    lib.stm_tuning_default.argtypes = [ctypes.POINTER(stm_tuning)]
+    lib.stm_tuning_default.restype = None
+    lib.stm_last_error.argtypes = []
+    lib.stm_last_error.restype = ctypes.c_char_p
+    return lib
+
+
+lib = _load()
+
+
+def _check(status: int) -> None:
+    if status != STM_OK:
+        raise StmError(status, lib.stm_last_error().decode())
+
+
+def _arr(a, dtype):
+    return None if a is None else np.ascontiguousarray(np.asarray(a, dtype=dtype))
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data
+
+
+# ---------------------------------------------------------------- same-name wrappers
+def stm_graph_load(n: int, row_ptr, col_idx, labels=None, device: int = 0) -> int:
+    rp, ci, lb = _arr(row_ptr, np.int64), _arr(col_idx, np.int32), _arr(labels, np.int32)
+    h = ctypes.c_void_p()
+    _check(lib.stm_graph_load(n, _p(rp), _p(ci), _p(lb), device, ctypes.byref(h)))
+    return h.value
+
+
+def stm_graph_load_device(n: int, nnz: int, d_row_ptr: int, d_col_idx: int, d_labels: Optional[int],
+                          device: int = 0) -> int:
+    h = ctypes.c_void_p()
+    _check(lib.stm_graph_load_device(n, nnz, d_row_ptr, d_col_idx, d_labels, device, ctypes.byref(h)))
+    return h.value
+
+
+def stm_graph_info(g: int) -> Tuple[int, int, int]:
+    n, nnz, md = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+    _check(lib.stm_graph_info(g, ctypes.byref(n), ctypes.byref(nnz), ctypes.byref(md)))
+    return n.value, nnz.value, md.value
+
+
+def stm_graph_free(g: int) -> None:
+    _check(lib.stm_graph_free(g))
+
+
+def stm_pattern_compile(k: int, edges, labels=None, order=None, restrictions=None, flags: int = 0) -> int:
+    e = _arr(edges, np.int32).reshape(-1)
+    lb = _arr(labels, np.int32)
+    od = _arr(order, np.int32)
+    rs = _arr(restrictions, np.int32).reshape(-1) if restrictions is not None and len(restrictions) else None
+    nr = 0 if rs is None else rs.size // 2
+    h = ctypes.c_void_p()
+    _check(lib.stm_pattern_compile(k, e.size // 2, _p(e), _p(lb), _p(od), nr, _p(rs), flags, ctypes.byref(h)))
+    return h.value
+
+
+def stm_plan_describe(p: int) -> str:
+    buf = ctypes.create_string_buffer(1 << 16)
+    _check(lib.stm_plan_describe(p, buf, len(buf)))
+    return buf.value.decode()
+
+
+def stm_plan_info(p: int) -> Tuple[int, int, int]:
+    k, ns, aut = ctypes.c_int(), ctypes.c_int(), ctypes.c_int64()
+    _check(lib.stm_plan_info(p, ctypes.byref(k), ctypes.byref(ns), ctypes.byref(aut)))
+    return k.value, ns.value, aut.value
+
+
+def stm_plan_first_vertex(p: int) -> int:
+    u = ctypes.c_int()
+    _check(lib.stm_plan_first_vertex(p, ctypes.byref(u)))
+    return u.value
+
+
+def stm_plan_free(p: int) -> None:
+    _check(lib.stm_plan_free(p))
+
+
+def stm_tuning_default(**overrides) -> stm_tuning:
+    t = stm_tuning()
+    lib.stm_tuning_default(ctypes.byref(t))
+    for k, v in overrides.items():
+        setattr(t, k, int(v))
+    return t
+
+
+def _tp(t: Optional[stm_tuning]):
+    return None if t is None else ctypes.cast(ctypes.pointer(t), ctypes.c_void_p)
+
+
+def make_shard(rank: int, world: int, chunk: int, cursor_ptrs: Sequence[Optional[int]]) -> stm_shard:
+    s = stm_shard()
+    s.rank, s.world, s.chunk = rank, world, chunk
+    for i, p in enumerate(cursor_ptrs):
+        s.d_cursors[i] = p
+    return s
+
+
+def stm_match_count(g: int, p: int, stream: Optional[int] = None) -> int:
+    c = ctypes.c_uint64()
+    _check(lib.stm_match_count(g, p, stream, ctypes.byref(c)))
+    return c.value
+
+
+def stm_match_count_ex(g: int, p: int, tuning: Optional[stm_tuning] = None, shard: Optional[stm_shard] = None,
+                       stream: Optional[int] = None) -> int:
+    c = ctypes.c_uint64()
+    sp = None if shard is None else ctypes.cast(ctypes.pointer(shard), ctypes.c_void_p)
+    _check(lib.stm_match_count_ex(g, p, _tp(tuning), sp, stream, ctypes.byref(c)))
+    return c.value
+
+
+def stm_match_count_async(g: int, p: int, d_count: int, tuning: Optional[stm_tuning] = None,
+                          shard: Optional[stm_shard] = None, stream: Optional[int] = None) -> None:
+    sp = None if shard is None else ctypes.cast(ctypes.pointer(shard), ctypes.c_void_p)
+    _check(lib.stm_match_count_async(g, p, _tp(tuning), sp, stream, d_count))
+
+
+def stm_match_count_per_root(g: int, p: int, tuning: Optional[stm_tuning] = None,
+                             stream: Optional[int] = None) -> Tuple[int, np.ndarray]:
+    n, _, _ = stm_graph_info(g)
+    out = np.zeros(max(n, 1), dtype=np.uint64)
+    c = ctypes.c_uint64()
+    _check(lib.stm_match_count_per_root(g, p, _tp(tuning), stream, out.ctypes.data, ctypes.byref(c)))
+    return c.value, out[:n]
+
+
+def stm_last_launch() -> dict:
+    info = stm_launch_info()
+    _check(lib.stm_last_launch(ctypes.byref(info)))
+    return {f[0]: getattr(info, f[0]) for f in info._fields_}
+
+
+# ---------------------------------------------------------------- convenience objects
+class Graph:
+    """Device-resident data graph (owns the stm_graph handle)."""
+
+    def __init__(self, n: int, row_ptr, col_idx, labels=None, device: int = 0):
+        self.handle = stm_graph_load(n, row_ptr, col_idx, labels, device)
+        self.n, self.nnz, self.max_degree = stm_graph_info(self.handle)
+        self.device = device
+
+    @classmethod
+    def from_stmgen(cls, g, device: int = 0) -> "Graph":
+        return cls(g.n, g.row_ptr, g.col_idx, g.labels, device)
+
+    def close(self):
+        if self.handle:
+            stm_graph_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Plan:
+    """Compiled pattern (owns the stm_plan handle)."""
+
+    def __init__(self, k: int, edges, labels=None, order=None, restrictions=None, vertex_induced=False,
+                 code_motion=True, auto_restrict=None, auto_order=False):
+        if auto_restrict is None:
+            auto_restrict = restrictions is None
+        flags = (STM_VERTEX_INDUCED if vertex_induced else 0) | (0 if code_motion else STM_NO_CODE_MOTION)
+        flags |= STM_AUTO_RESTRICT if auto_restrict else 0
+        flags |= STM_AUTO_ORDER if auto_order else 0
+        self.handle = stm_pattern_compile(k, edges, labels, order, restrictions, flags)
+        self.k, self.n_sets, self.aut = stm_plan_info(self.handle)
+        self.first_vertex = stm_plan_first_vertex(self.handle)
+
+    @classmethod
+    def from_pattern(cls, p, **kw) -> "Plan":
+        return cls(p.k, p.edges, p.labels, **kw)
+
+    def describe(self) -> str:
+        return stm_plan_describe(self.handle)
+
+    def close(self):
+        if self.handle:
+            stm_plan_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def count(graph: Graph, plan: Plan, tuning: Optional[stm_tuning] = None, stream: Optional[int] = None) -> int:
+    return stm_match_count_ex(graph.handle, plan.handle, tuning, None, stream)

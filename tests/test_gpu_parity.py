@@ -1,0 +1,211 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle, bit-exact.
+
+Every count here is an exact integer; the bar is equality.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import oracle
+import stmgen
+from stmgen import CATALOG
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover - CPU container
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_sc_weij22_b200 import stm  # noqa: E402  (fails loudly if libstm.so is missing)
+
+SMALL = ["edge", "wedge", "triangle", "path4", "star4", "c4", "diamond", "tailed_triangle", "k4",
+         "house", "c5", "k5"]
+BIG = ["k6", "k6_minus_e", "octahedron", "w5", "prism", "c6", "k7_minus_e", "w6", "c7"]
+
+
+def ocount(g, p, vi, labels=None, restr="auto", threads=0):
+    R = oracle.gk_restrictions(p.k, p.edges, labels) if restr == "auto" else restr
+    return oracle.count(g, p.k, p.edges, plabels=labels, vertex_induced=vi, restrictions=R,
+                        threads=threads)
+
+
+def gcount(G, p, vi, labels=None, restr="auto", tuning=None, **kw):
+    if restr == "auto":
+        plan = stm.Plan(p.k, p.edges, labels, vertex_induced=vi, **kw)
+    else:
+        plan = stm.Plan(p.k, p.edges, labels, restrictions=restr, auto_restrict=False, vertex_induced=vi, **kw)
+    return stm.count(G, plan, tuning)
+
+
+@pytest.fixture(scope="module")
+def er_small():
+    g = stmgen.er(300, 2500, 7)
+    g.labels = stmgen.labels(g.n, 3, 8)
+    return g, stm.Graph.from_stmgen(g)
+
+
+@pytest.fixture(scope="module")
+def er_sparse():
+    g = stmgen.er(300, 1500, 9)
+    return g, stm.Graph.from_stmgen(g)
+
+
+@pytest.fixture(scope="module")
+def rmat_small():
+    # hubs (max degree ~250 of 1024 vertices) so that stealing and long/short operands mix
+    g = stmgen.rmat(10, 4000, 0.57, 0.19, 0.19, 17)
+    g.labels = stmgen.labels(g.n, 4, 18)
+    return g, stm.Graph.from_stmgen(g)
+
+
+@pytest.mark.parametrize("name", SMALL)
+@pytest.mark.parametrize("vi", [False, True])
+def test_small_patterns_er(er_small, name, vi):
+    g, G = er_small
+    p = CATALOG[name]
+    assert gcount(G, p, vi) == ocount(g, p, vi)
+
+
+@pytest.mark.parametrize("name", SMALL + ["k6", "k6_minus_e", "k7_minus_e", "octahedron"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_patterns_rmat_hubs(rmat_small, name, vi):
+    g, G = rmat_small
+    p = CATALOG[name]
+    assert gcount(G, p, vi) == ocount(g, p, vi)
+
+
+@pytest.mark.parametrize("name", ["w5", "prism", "c6", "c7", "w6", "k8"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_size6_8_sparse(er_sparse, name, vi):
+    g, G = er_sparse
+    p = CATALOG[name]
+    assert gcount(G, p, vi) == ocount(g, p, vi)
+
+
+def test_size6_7_hubs_vertex_induced(rmat_small):
+    g, G = rmat_small
+    for name in ["w5", "prism", "c6"]:
+        p = CATALOG[name]
+        assert gcount(G, p, True) == ocount(g, p, True), name
+
+
+@pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "house", "c5", "k4", "tailed_triangle"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_labeled(rmat_small, name, vi):
+    g, G = rmat_small
+    p = CATALOG[name]
+    rng = np.random.default_rng(hash(name) % 1000)
+    for _ in range(3):
+        pl = tuple(int(x) for x in rng.integers(0, 4, p.k))
+        assert gcount(G, p, vi, pl) == ocount(g, p, vi, pl)
+
+
+@pytest.mark.parametrize("name", ["c4", "house", "diamond", "path4", "c5"])
+def test_unrestricted_and_custom_restrictions(er_small, name):
+    g, G = er_small
+    p = CATALOG[name]
+    for vi in (False, True):
+        assert gcount(G, p, vi, restr=[]) == ocount(g, p, vi, restr=[])
+        R = [(1, 0)] if p.k > 1 else []
+        assert gcount(G, p, vi, restr=R) == ocount(g, p, vi, restr=R)
+
+
+TUNINGS = [
+    dict(local_steal=0, global_steal=0),
+    dict(local_steal=1, global_steal=0),
+    dict(local_steal=1, global_steal=1),
+    dict(local_steal=0, global_steal=1),
+    dict(unroll=1), dict(unroll=2), dict(unroll=16),
+    dict(root_chunk=1, stop_level=3, detect_level=3),
+    dict(block_warps=4), dict(block_warps=32, blocks_per_sm=1),
+]
+
+
+@pytest.mark.parametrize("tk", range(len(TUNINGS)))
+def test_tuning_invariance(rmat_small, tk):
+    """Every scheduler switch (ablation of Fig. 12) leaves the count unchanged."""
+    g, G = rmat_small
+    t = stm.stm_tuning_default(**TUNINGS[tk])
+    for name, vi in [("k4", False), ("house", True), ("c5", False), ("diamond", True), ("triangle", False)]:
+        p = CATALOG[name]
+        assert gcount(G, p, vi, tuning=t) == ocount(g, p, vi), (name, vi, TUNINGS[tk])
+
+
+@pytest.mark.parametrize("name", ["house", "diamond", "c5", "k5", "prism"])
+def test_code_motion_and_order_invariance(rmat_small, name):
+    g, G = rmat_small
+    p = CATALOG[name]
+    for vi in (False, True):
+        want = ocount(g, p, vi)
+        assert gcount(G, p, vi, code_motion=False) == want
+        for perm in list(itertools.permutations(range(p.k)))[:: max(1, len(list(itertools.permutations(range(p.k)))) // 6)]:
+            adj = {u: set() for u in range(p.k)}
+            for a, b in p.edges:
+                adj[a].add(b)
+                adj[b].add(a)
+            if all(any(perm[j] in adj[perm[i]] for j in range(i)) for i in range(1, p.k)):
+                assert gcount(G, p, vi, order=list(perm)) == want
+
+
+def test_golden_config_counts():
+    """Full-size config graphs against stored oracle counts (tools/make_golden.py,
+    fingerprints checked so the very same graph is compared)."""
+    import json, os
+    path = os.path.join(os.path.dirname(__file__), "golden", "config_counts.json")
+    data = json.load(open(path))
+    graphs = {}
+    for cid, d in sorted(data.items()):
+        if d["config"] not in graphs:
+            g = stmgen.config_graph(d["config"])
+            graphs[d["config"]] = (g, stm.Graph.from_stmgen(g))
+        g, G = graphs[d["config"]]
+        assert g.fingerprint() == d["fingerprint"], cid
+        plan = stm.Plan(d["k"], d["edges"], d["labels"], restrictions=d["restrictions"], auto_restrict=False,
+                        vertex_induced=d["vertex_induced"])
+        assert stm.count(G, plan) == d["count"], cid
+        plan2 = stm.Plan(d["k"], d["edges"], d["labels"], vertex_induced=d["vertex_induced"])
+        assert stm.count(G, plan2) == d["count"], cid + " (compiler's own restrictions)"
+
+
+@pytest.mark.parametrize("cfg,name,ntop", [("c2", "k4", 1), ("c2", "c4", 0), ("c3", "house", 0), ("c5", "k5", 1),
+                                           ("c3", "k5", 0)])
+def test_config_scale_sampled_roots(cfg, name, ntop):
+    """At full size, in the bench's launch configuration: GPU per-root counts on a
+    sample of roots (random + the highest-degree ones) equal the oracle's."""
+    g = stmgen.config_graph(cfg)
+    G = stm.Graph.from_stmgen(g)
+    p = CATALOG[name]
+    plan = stm.Plan(p.k, p.edges)
+    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
+    assert int(pr.sum(dtype=np.uint64)) == tot
+    rng = np.random.default_rng(5)
+    deg = g.degrees()
+    top = np.argsort(deg)[len(deg) - ntop:] if ntop else np.zeros(0, np.int64)
+    roots = np.unique(np.concatenate([rng.choice(g.n, 48, replace=False), top]))
+    R = oracle.gk_restrictions(p.k, p.edges)
+    oc, opr = oracle.count(g, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=roots, per_root=True)
+    assert np.array_equal(pr[roots], opr)
+
+
+def test_degenerate_graphs():
+    for g in [stmgen.complete(8), stmgen.cycle(7), stmgen.grid(4, 5), stmgen.empty(5)]:
+        G = stm.Graph.from_stmgen(g)
+        for name in ["triangle", "c4", "k4", "c6", "c7", "house"]:
+            p = CATALOG[name]
+            for vi in (False, True):
+                assert gcount(G, p, vi) == ocount(g, p, vi), (g.name, name, vi)
+
+
+def test_per_root_histogram(rmat_small):
+    """Localisation: GPU per-root counts equal the oracle's, attributed to f(order[0])."""
+    g, G = rmat_small
+    for name, vi in [("diamond", False), ("house", True), ("k4", False)]:
+        p = CATALOG[name]
+        plan = stm.Plan(p.k, p.edges, vertex_induced=vi)
+        tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(root_chunk=1))
+        R = oracle.gk_restrictions(p.k, p.edges)
+        otot, opr = oracle.count(g, p.k, p.edges, vertex_induced=vi, restrictions=R,
+                                 root_u=plan.first_vertex, per_root=True)
+        assert tot == otot
+        assert np.array_equal(pr, opr)
