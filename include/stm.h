@@ -143,7 +143,9 @@ typedef struct stm_tuning {
   int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 32. */
   int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
-  int32_t debug_per_root; /* 2 = instrumented launch: count algorithmic bytes (stm_last_launch); else reserved */
+  int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
+  int32_t hash_slots;     /* per-warp shared-memory hash set for operands shared by a combined set
+                             operation: 0 = off, else a power of two in 64..4096 slots. Default 0. */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -213,7 +215,7 @@ typedef struct stm_launch_info {
   int64_t local_steals;    /* intra-block steals (Sec. V-A); synchronous calls only */
   int64_t global_steals;   /* inter-block steals (Sec. V-B); synchronous calls only */
   int64_t chunks;          /* root chunks taken from cursors; synchronous calls only */
-  int64_t alg_bytes;       /* algorithmic bytes W; instrumented calls only (tuning.debug_per_root == 2) */
+  int64_t alg_bytes;       /* algorithmic bytes W; instrumented calls only (tuning.instrument == 1) */
   int64_t merge_bytes;     /* merge-equivalent bytes W_merge; instrumented calls only */
   int64_t jobs;            /* set operations executed; instrumented calls only */
 } stm_launch_info;

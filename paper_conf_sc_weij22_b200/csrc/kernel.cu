@@ -24,8 +24,11 @@
 // PAPER.md:84) and inter-block stealing through per-block global mailboxes pushed
 // by busy donors (Sec. V-B, Fig. 6).  Stolen work is a task
 // (prefix, position range); the thief rebuilds the prefix's sets itself.
+#include <algorithm>
 #include <climits>
+#include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 
 #include <cuda_runtime.h>
@@ -33,6 +36,7 @@
 #include "kernel.h"
 
 #define FULLMASK 0xffffffffu
+#define HT_MIN 16
 
 namespace {
 
@@ -43,6 +47,7 @@ struct WarpHdr {
   int nsib[STM_KMAX], cur[STM_KMAX], it[STM_KMAX], end[STM_KMAX];
   int used[STM_MAX_NODES];    // words used in each node region by the frame being built
   int stage_c[32], stage_u[32];
+  unsigned lgen[STM_KMAX + 1];  // per-level generation of the arena set nodes
 };
 
 struct BlockHdr {
@@ -54,8 +59,8 @@ struct BlockHdr {
 };
 
 __host__ __device__ constexpr int warp_bytes_fixed() { return (int)sizeof(WarpHdr); }
-__host__ __device__ inline int warp_bytes(int k, int n_nodes) {
-  int b = warp_bytes_fixed() + k * STM_RMAX * 4 + 2 * n_nodes * STM_UMAX * 4;
+__host__ __device__ inline int warp_bytes(int k, int n_nodes, int ht_slots) {
+  int b = warp_bytes_fixed() + k * STM_RMAX * 4 + 2 * n_nodes * STM_UMAX * 4 + ht_slots * 4;
   return (b + 15) & ~15;
 }
 
@@ -72,7 +77,14 @@ struct W {
   unsigned exhausted;  // cursors known to be exhausted (bit per rank)
   unsigned long long cnt;
   unsigned gather_calls;
+  unsigned donate_tick;
+  int steal_fails;
   unsigned long long wbytes, wmerge, wjobs;  // per-lane instrumentation partials
+  int* ht;                          // shared-memory hash set (HT_SLOTS ints)
+  unsigned ht_mask;
+  unsigned long long ht_ptr;        // key of the hashed operand
+  int ht_len;
+  unsigned ht_gen;                  // lgen of the hashed node's level when it was hashed
 };
 
 #define SIB(w, l, u) ((w).sib[(l) * STM_RMAX + (u)])
@@ -142,6 +154,43 @@ __device__ __forceinline__ bool labok(const W& w, int x, unsigned lab) {
 }
 
 // ----------------------------------------------------------------------------
+// Per-warp shared-memory hash set of one sorted operand (B200 design choice, see
+// DESIGN.md "Kernel"): when every job of a combined operation shares an operand
+// (a set of the current DFS path, e.g. N(v0) for all level-2 jobs of a root), it
+// is hashed once into the warp's shared-memory table and every membership probe
+// becomes ~1 shared-memory load instead of a binary search through L1/L2.  The
+// table stays valid while the same operand is reused by later operations.
+// ----------------------------------------------------------------------------
+__device__ __forceinline__ unsigned ht_hash(int x, unsigned mask) {
+  return (((unsigned)x * 0x9E3779B1u) >> 7) & mask;
+}
+
+__device__ __noinline__ void ht_build(W& w, const int* a, int n) {
+  unsigned size = 64;
+  while (size < 2u * (unsigned)n) size <<= 1;
+  const unsigned mask = size - 1;
+  for (unsigned i = w.lane; i < size; i += 32) w.ht[i] = -1;
+  __syncwarp();
+  for (int i = w.lane; i < n; i += 32) {
+    const int x = a[i];
+    unsigned h = ht_hash(x, mask);
+    while (atomicCAS(&w.ht[h], -1, x) != -1) h = (h + 1) & mask;
+  }
+  __syncwarp();
+  w.ht_mask = mask;
+}
+
+__device__ __forceinline__ bool ht_has(const int* ht, unsigned mask, int x) {
+  unsigned h = ht_hash(x, mask);
+  for (;;) {
+    const int v = ht[h];
+    if (v == x) return true;
+    if (v < 0) return false;
+    h = (h + 1) & mask;
+  }
+}
+
+// ----------------------------------------------------------------------------
 // Flattened multi-job set operation (Fig. 8).  Lane j < njobs owns job j.
 // ----------------------------------------------------------------------------
 struct Job {
@@ -153,36 +202,96 @@ struct Job {
   unsigned lab;
   int* out;      // materialise target (NULL in count mode)
   int u, c;      // context for exclusions / per-root attribution
+  int a_node;    // 0: A is a CSR row; l+1: A is an arena set node of level l (rebuilt with its frame)
 };
+
+__device__ __forceinline__ void narrow(const int*& p, int& n, int lo, int hi) {
+  if (n > 16) {
+    if (lo >= 0) { int b = lbound(p, n, lo + 1); p += b; n -= b; }
+    if (hi < INT_MAX) n = lbound(p, n, hi);
+  }
+}
+
+__device__ __forceinline__ int log2c(int n) { return 32 - __clz(n); }  // ceil(log2(n+1))
 
 // Returns the (warp-uniform) number of kept elements summed over all jobs when
 // counting; in materialise mode *outc (lane j) receives job j's output size.
-__device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F, unsigned excl,
-                                       int* outc_lane) {
+__device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F,
+                                                    unsigned excl, int* outc_lane) {
   const int lane = w.lane;
   const bool mine = lane < njobs;
-  const int* D = J.A;
-  const int* Pp = J.B;
-  int dlen = J.alen, plen = J.B ? J.blen : 0;
-  if (mine && J.op == STM_OP_AND && J.blen < J.alen) {
-    D = J.B; dlen = J.blen; Pp = J.A; plen = J.alen;
+  // operands narrowed to the open interval (lo, hi) of the restriction bounds
+  const int* An = J.A;
+  int an = mine ? J.alen : 0;
+  const int* Bn = J.B;
+  int bn = (mine && J.B) ? J.blen : 0;
+  if (mine) {
+    narrow(An, an, J.lo, J.hi);
+    if (J.B) narrow(Bn, bn, J.lo, J.hi);
   }
-  if (!mine) dlen = 0;
-  if (mine) {  // narrow both operands to the open interval (lo, hi)
-    if (dlen > 16) {
-      if (J.lo >= 0) { int b = lbound(D, dlen, J.lo + 1); D += b; dlen -= b; }
-      if (J.hi < INT_MAX) dlen = lbound(D, dlen, J.hi);
+  // ---- shared operand -> shared-memory hash set
+  const unsigned long long a0 = __shfl_sync(FULLMASK, (unsigned long long)J.A, 0);
+  const unsigned long long b0 = __shfl_sync(FULLMASK, (unsigned long long)J.B, 0);
+  const int al0 = __shfl_sync(FULLMASK, J.alen, 0), bl0 = __shfl_sync(FULLMASK, J.blen, 0);
+  const int op0 = __shfl_sync(FULLMASK, J.op, 0);
+  const bool sameA = __all_sync(FULLMASK, !mine || ((unsigned long long)J.A == a0 && J.alen == al0 && J.op == STM_OP_AND));
+  const bool sameB = __all_sync(FULLMASK, !mine || ((unsigned long long)J.B == b0 && J.blen == bl0 && J.B != nullptr));
+  int hmode = 0;  // 1: A hashed (drive B), 2: B hashed (drive A)
+  const int* hp = nullptr;
+  int hn = 0;
+  int hnode = 0;
+  const int ht_max = w.kp->ht_slots / 2;
+  if (sameA && al0 >= HT_MIN && al0 <= ht_max && b0 != 0ull) {  // (warp-uniform: lane 0 owns a job)
+    hmode = 1; hp = (const int*)a0; hn = al0; hnode = __shfl_sync(FULLMASK, J.a_node, 0);
+  } else if (sameB && bl0 >= HT_MIN && bl0 <= ht_max) {
+    hmode = 2; hp = (const int*)b0; hn = bl0;
+  }
+  if (hmode) {
+    const unsigned g = hnode ? w.h->lgen[hnode - 1] : 0u;
+    const bool cached = (unsigned long long)hp == w.ht_ptr && hn == w.ht_len && w.ht_gen == g;
+    if (!cached) {
+      // build only if the probes it saves outweigh the build (~ table size + 2n lane-ops)
+      int save = 0;
+      if (mine) {
+        const int dh = hmode == 1 ? bn : an;  // driven elements in hash mode
+        int d, pl;
+        if (J.op == STM_OP_AND) { d = min(an, bn); pl = max(an, bn); } else { d = an; pl = bn; }
+        save = max(0, d * (log2c(pl) + 1) * 4 - dh * 2);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) save += __shfl_xor_sync(FULLMASK, save, o);
+      if (save > 4 * hn + 128) {
+        ht_build(w, hp, hn);
+        w.ht_ptr = (unsigned long long)hp;
+        w.ht_len = hn;
+        w.ht_gen = g;
+      } else {
+        hmode = 0;
+      }
     }
-    if (plen > 16) {
-      if (J.lo >= 0) { int b = lbound(Pp, plen, J.lo + 1); Pp += b; plen -= b; }
-      if (J.hi < INT_MAX) plen = lbound(Pp, plen, J.hi);
+  }
+  // ---- per-job driving side: 0 = binary search, 1 = hash probe
+  const int* D = An;
+  const int* Pp = Bn;
+  int dlen = an, plen = bn, use_h = 0;
+  if (mine) {
+    if (J.op == STM_OP_AND && bn < an) { D = Bn; dlen = bn; Pp = An; plen = an; }
+    if (!J.B) { Pp = nullptr; plen = 0; }
+    if (hmode) {
+      const int dh = hmode == 1 ? bn : an;
+      if (dh * 2 <= dlen * (log2c(plen) + 1) * 4) {
+        use_h = 1;
+        if (hmode == 1) { D = Bn; dlen = bn; } else { D = An; dlen = an; }
+      }
     }
   }
   if (w.kp->count_bytes && mine) {
-    // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below)
-    const long long lg = 32 - __clz(plen);  // ceil(log2(plen+1))
-    w.wbytes += 4ull * (unsigned long long)dlen + 4ull * (unsigned long long)min((long long)plen, (long long)dlen * lg);
-    w.wmerge += 4ull * (unsigned long long)(dlen + plen);
+    // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below),
+    // with A the driving operand and B the probed one (before hashing).
+    int d, pl;
+    if (J.op == STM_OP_AND) { d = min(an, bn); pl = max(an, bn); } else { d = an; pl = bn; }
+    w.wbytes += 4ull * (unsigned long long)d + 4ull * (unsigned long long)min((long long)pl, (long long)d * log2c(pl));
+    w.wmerge += 4ull * (unsigned long long)(an + bn);
     w.wjobs += 1;
   }
   int incl = dlen;
@@ -193,7 +302,11 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
   }
   const int total = __shfl_sync(FULLMASK, incl, 31);
   const int start = incl - dlen;
-  const bool has_p = Pp != nullptr;
+  const int flags = (Pp != nullptr ? 1 : 0) | (use_h ? 2 : 0) | (J.op == STM_OP_DIFF ? 4 : 0);
+  const int* const ht = w.ht;
+  const unsigned htmask = w.ht_mask;
+  const uint8_t* const glabels = w.kp->labels;
+  const unsigned char* const l2s = w.bh->lab2slot;
   int outc = 0;
   unsigned long long jc = 0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
@@ -211,21 +324,20 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
     const int* Pj = (const int*)__shfl_sync(FULLMASK, Pll, j);
     const int sj = __shfl_sync(FULLMASK, start, j);
     const int pl = __shfl_sync(FULLMASK, plen, j);
-    const int opj = __shfl_sync(FULLMASK, J.op, j);
+    const int fj = __shfl_sync(FULLMASK, flags, j);
     const int loj = __shfl_sync(FULLMASK, J.lo, j);
     const int hij = __shfl_sync(FULLMASK, J.hi, j);
     const unsigned labj = __shfl_sync(FULLMASK, J.lab, j);
-    const int hp = __shfl_sync(FULLMASK, (int)has_p, j);
     bool keep = false;
     int x = 0;
     if (valid) {
       x = Dj[e - sj];
       keep = x > loj && x < hij;
-      if (keep && hp) {
-        bool f = member(Pj, pl, x);
-        keep = (opj == STM_OP_DIFF) ? !f : f;
+      if (keep && (fj & 1)) {
+        const bool f = (fj & 2) ? ht_has(ht, htmask, x) : member(Pj, pl, x);
+        keep = (fj & 4) ? !f : f;
       }
-      if (keep) keep = labok(w, x, labj);
+      if (keep && labj != STM_LAB_ANY) keep = (l2s[glabels[x]] & labj) != 0;
     }
     const unsigned km = __ballot_sync(FULLMASK, keep);
     // lanes of my own job inside this chunk
@@ -289,6 +401,7 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   J.out = nullptr;
   J.u = u;
   J.c = c;
+  J.a_node = P.cnt_a.kind == STM_SRC_NODE ? P.nodes[P.cnt_a.idx].level + 1 : 0;
   return J;
 }
 
@@ -370,6 +483,8 @@ __device__ void build_nodes(W& w, int F, int m) {
   const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
   if (nb == ne) return;
   const int u = F >= 1 ? w.h->cur[F] : 0;
+  if (w.lane == 0) w.h->lgen[F + 1] += 1;  // level F+1 sets are overwritten: drop stale hashes
+  __syncwarp();
   for (int st = 0; st < P.n_stages[F + 1]; ++st) {
     // jobs of this stage: (node, sibling) pairs
     int nodes_in[STM_MAX_NODES];
@@ -382,7 +497,7 @@ __device__ void build_nodes(W& w, int F, int m) {
       const int nj = min(32, njobs_total - j0);
       Job J;
       J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_AND;
-      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0;
+      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0;
       int s = 0, t = 0;
       if (w.lane < nj) {
         s = nodes_in[jj / m];
@@ -392,6 +507,7 @@ __device__ void build_nodes(W& w, int F, int m) {
         J.c = c;
         if (nd.a_kind == STM_SRC_RAW) row(w, pval(w, nd.a, F, u, c), J.A, J.alen);
         else node_slice(w, nd.a, F, u, t, J.A, J.alen);
+        J.a_node = nd.a_kind == STM_SRC_NODE ? P.nodes[nd.a].level + 1 : 0;
         row(w, pval(w, nd.b, F, u, c), J.B, J.blen);
         J.op = nd.op;
         bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
@@ -534,7 +650,7 @@ __device__ void frame_count(W& w, int m) {
   const int u = F >= 1 ? w.h->cur[F] : 0;
   Job J;
   J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
-  J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0;
+  J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0;
   if (w.lane < m) J = count_job(w, F, u, SIB(w, k - 1, w.lane), w.lane);
   w.cnt += run_jobs(w, J, m, true, F, w.P->filt[k - 1].excl, nullptr);
 }
@@ -595,7 +711,7 @@ __device__ void fused_count(W& w, int F) {
     if (nj == 0) return;
     Job J;
     J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
-    J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0;
+    J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0; J.a_node = 0;
     if (w.lane < nj) J = count_job(w, F, w.h->stage_u[w.lane], w.h->stage_c[w.lane], 0);
     w.cnt += run_jobs(w, J, nj, true, F, P.filt[P.k - 1].excl, nullptr);
     __syncwarp();
@@ -605,7 +721,7 @@ __device__ void fused_count(W& w, int F) {
 // ----------------------------------------------------------------------------
 // work acquisition: root chunks, local steal, global steal (Sec. V)
 // ----------------------------------------------------------------------------
-__device__ bool try_chunk(W& w) {
+__device__ __noinline__ bool try_chunk(W& w) {
   const StmKParams& kp = *w.kp;
   int b = -1, e = -1;
   if (w.lane == 0) {
@@ -638,65 +754,72 @@ __device__ bool try_chunk(W& w) {
   return true;
 }
 
-// Split the stack of `v` (caller holds v's lock).  Takes half of the shallowest
-// stealable remaining work.  Work at the victim's current
-// frame L is not in progress yet, so there the victim always keeps at least one
-// item (otherwise a single item could be passed around forever); at frames
-// shallower than L the victim is busy below and the thief may take it all.
-// Returns false if nothing can be taken.
-__device__ bool split_stack(const W& w, volatile WarpHdr* v, volatile int* vsib, StmTask& T) {
+// What a steal from stack `v` would take (half of the
+// shallowest stealable remaining work).  Work at the victim's current frame L is
+// not in progress yet, so there the victim always keeps at least one item
+// (otherwise a single item could be passed around forever); at frames shallower
+// than L the victim is busy below and the thief may take it all.
+// kind: 0 = root range of frame 0, 1 = remaining root siblings of frame 1,
+// 2 = remaining candidates of the current sibling of frame F.  F < 0: nothing.
+struct SplitPick {
+  int F, kind, t;
+};
+
+__device__ __forceinline__ SplitPick pick_split(const W& w, volatile WarpHdr* v) {
   const int L = v->L;
-  // frame 0: root range
-  int r = v->root_end - v->root_it;
-  int t = (L > 0) ? (r + 1) / 2 : r / 2;
-  if (t >= 1) {
-    T.level = 0;
-    T.e = v->root_end;
-    T.b = v->root_end - t;
-    v->root_end = T.b;
-    return true;
-  }
+  const int r = v->root_end - v->root_it;
+  const int t = (L > 0) ? (r + 1) / 2 : r / 2;
+  if (t >= 1) return {0, 0, t};
   const int stop = w.kp->stop_level;
   for (int F = 1; F <= L && F < stop; ++F) {
-    if (v->cur[F] >= v->nsib[F]) continue;
+    const int cur = v->cur[F], nsib = v->nsib[F];
+    if (cur >= nsib) continue;
     const int rem = v->end[F] - v->it[F];
-    if (F == 1) {  // remaining root siblings -> root range
-      int rs = v->nsib[1] - v->cur[1] - 1;
-      int ts = (L > 1 || rem > 0) ? (rs + 1) / 2 : rs / 2;
-      if (ts >= 1) {
-        int s0 = v->nsib[1] - ts;
-        T.level = 0;
-        T.b = vsib[1 * STM_RMAX + s0];
-        T.e = vsib[1 * STM_RMAX + v->nsib[1] - 1] + 1;
-        v->nsib[1] = s0;
-        return true;
-      }
+    if (F == 1) {
+      const int rs = nsib - cur - 1;
+      const int ts = (L > 1 || rem > 0) ? (rs + 1) / 2 : rs / 2;
+      if (ts >= 1) return {1, 1, ts};
     }
-    const bool last_sib = v->cur[F] + 1 >= v->nsib[F];
+    const bool last_sib = cur + 1 >= nsib;
     const int tr = (L > F || !last_sib) ? (rem + 1) / 2 : rem / 2;
-    if (tr >= 1) {
-      T.level = F;
-      T.e = v->end[F];
-      T.b = v->end[F] - tr;
-      for (int j = 0; j < F; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1]];
-      v->end[F] = T.b;
-      return true;
-    }
+    if (tr >= 1) return {F, 2, tr};
   }
-  return false;
+  return {-1, 0, 0};
 }
 
-// crude amount-of-work score of a stack (higher = better victim), racy read
-__device__ int steal_score(const W& w, volatile WarpHdr* v) {
-  if (v->root_end - v->root_it >= 1) return 1 << 30;
-  const int L = v->L;
-  for (int F = 1; F <= L && F < w.kp->stop_level; ++F) {
-    int rs = (F == 1) ? v->nsib[1] - v->cur[1] - 1 : 0;
-    int rem = v->end[F] - v->it[F];
-    if (v->cur[F] >= v->nsib[F]) rem = 0;
-    if (rs > 0 || rem > 0) return ((STM_KMAX - F) << 24) + min(rs * 1024 + rem, (1 << 24) - 1);
+// Split the stack of `v` (caller holds v's lock).  Returns false if nothing.
+__device__ __noinline__ bool split_stack(const W& w, volatile WarpHdr* v, volatile int* vsib, StmTask& T) {
+  const SplitPick s = pick_split(w, v);
+  if (s.F < 0) return false;
+  if (s.kind == 0) {
+    T.level = 0;
+    T.e = v->root_end;
+    T.b = v->root_end - s.t;
+    v->root_end = T.b;
+  } else if (s.kind == 1) {  // remaining root siblings -> root range
+    const int s0 = v->nsib[1] - s.t;
+    T.level = 0;
+    T.b = vsib[1 * STM_RMAX + s0];
+    T.e = vsib[1 * STM_RMAX + v->nsib[1] - 1] + 1;
+    v->nsib[1] = s0;
+  } else {
+    const int F = s.F;
+    T.level = F;
+    T.e = v->end[F];
+    T.b = v->end[F] - s.t;
+    for (int j = 0; j < F; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1]];
+    v->end[F] = T.b;
   }
-  return 0;
+  return true;
+}
+
+// amount-of-work score of a stack (higher = better victim; 0 = nothing a split
+// would take), racy read without the lock
+__device__ __forceinline__ int steal_score(const W& w, volatile WarpHdr* v) {
+  const SplitPick s = pick_split(w, v);
+  if (s.F < 0) return 0;
+  if (s.F == 0) return 1 << 30;
+  return ((STM_KMAX - s.F) << 24) + min(s.t * (s.kind == 1 ? 1024 : 1), (1 << 24) - 1);
 }
 
 __device__ volatile WarpHdr* warp_hdr(const W& w, int wid);
@@ -719,7 +842,7 @@ __device__ volatile int* warp_sib(const W& w, int wid);
 
 // Rebuild this warp's stack from a task (the receiver recomputes the sets of
 // levels 1..T.level from the prefix).
-__device__ void adopt_task(W& w, const StmTask& T) {
+__device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   const int k = w.P->k;
   if (T.level == 0) {
     lock_ws(w, w.h);
@@ -759,7 +882,7 @@ __device__ void adopt_task(W& w, const StmTask& T) {
   unlock_ws(w, w.h);
 }
 
-__device__ bool try_local_steal(W& w) {
+__device__ __noinline__ bool try_local_steal(W& w) {
   const int nw = w.kp->block_warps;
   // pick the best victim (racy scores), then split under its lock
   int best = -1, bs = 0;
@@ -793,16 +916,21 @@ __device__ bool try_local_steal(W& w) {
 }
 
 // donor side of Fig. 6: give half of my shallowest work to an idle block
-__device__ void maybe_donate(W& w) {
+__device__ __noinline__ void maybe_donate(W& w) {
   const StmKParams& kp = *w.kp;
+  // the idle-block count lives in L2: look at it on every 8th opportunity only
+  if ((++w.donate_tick & (unsigned)w.kp->donate_mask) != 0) return;
   int idle = 0;
   if (w.lane == 0) idle = *(volatile int*)&kp.work->idle_blocks;
   idle = bcast(idle);
   if (idle <= 0) return;
+  // only donate what a split can actually take
+  if (pick_split(w, w.h).F < 0) return;
   const int nb = gridDim.x;
   int target = -1;
-  for (int b0 = 0; b0 < nb && target < 0; b0 += 32) {
-    int b = (blockIdx.x + 1 + b0 + w.lane) % nb;
+  const int off = (int)((blockIdx.x * 37u + w.wid * 11u + w.donate_tick) % (unsigned)nb);
+  for (int b0 = 0; b0 < min(nb, 64) && target < 0; b0 += 32) {
+    int b = (off + b0 + w.lane) % nb;
     bool cand = (b0 + w.lane < nb) && b != (int)blockIdx.x &&
                 *(volatile int*)&kp.slots[b].is_idle == 1;
     unsigned cm = __ballot_sync(FULLMASK, cand);
@@ -841,7 +969,7 @@ __device__ void maybe_donate(W& w) {
 }
 
 // No more local work: returns true with new work adopted, false on termination.
-__device__ bool acquire_work(W& w, long long t0) {
+__device__ __noinline__ bool acquire_work(W& w, long long t0) {
   const StmKParams& kp = *w.kp;
   if (try_chunk(w)) return true;
   if (!kp.local_steal && !kp.global_steal) return false;
@@ -925,7 +1053,8 @@ __device__ bool acquire_work(W& w, long long t0) {
       // while a stolen task is in flight
       if (w.lane == 0) atomicAnd(&bh->idle_mask, (int)~me);
       __syncwarp();
-      if (try_local_steal(w)) return true;
+      if (try_local_steal(w)) { w.steal_fails = 0; return true; }
+      w.steal_fails = min(w.steal_fails + 1, w.kp->backoff_max);
       if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
       old = bcast(old);
       if ((((unsigned)old) | me) == all) {
@@ -933,14 +1062,14 @@ __device__ bool acquire_work(W& w, long long t0) {
         __syncwarp();
       }
     }
-    if (w.lane == 0) __nanosleep(spin < 64 ? 64 : 512);
+    if (w.lane == 0) __nanosleep(32u << w.steal_fails);  // back off while nothing can be stolen
     __syncwarp();
   }
 }
 
 __device__ volatile WarpHdr* warp_hdr(const W& w, int wid) {
   extern __shared__ __align__(16) unsigned char smem[];
-  int wb = warp_bytes(w.P->k, w.P->n_nodes);
+  int wb = warp_bytes(w.P->k, w.P->n_nodes, w.kp->ht_slots);
   return (volatile WarpHdr*)(smem + sizeof(BlockHdr) + (size_t)wid * wb);
 }
 __device__ volatile int* warp_sib(const W& w, int wid) {
@@ -963,7 +1092,7 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
     bh->done = 0;
   }
   for (int i = threadIdx.x; i < 256; i += blockDim.x) bh->lab2slot[i] = kp.lab2slot[i];
-  const int wb = warp_bytes(P.k, P.n_nodes);
+  const int wb = warp_bytes(P.k, P.n_nodes, kp.ht_slots);
   unsigned char* wbase = smem + sizeof(BlockHdr) + (size_t)wid * wb;
   W w;
   w.kp = &kp;
@@ -972,6 +1101,11 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
   w.sib = (volatile int*)(wbase + sizeof(WarpHdr));
   w.noff = (int*)(wbase + sizeof(WarpHdr) + P.k * STM_RMAX * 4);
   w.nsz = w.noff + P.n_nodes * STM_UMAX;
+  w.ht = w.nsz + P.n_nodes * STM_UMAX;
+  w.ht_mask = 0;
+  w.ht_ptr = 0;
+  w.ht_len = -1;
+  w.ht_gen = 0;
   w.bh = bh;
   const long long gw = (long long)blockIdx.x * kp.block_warps + wid;
   w.arena = kp.arena + (size_t)gw * (size_t)P.n_nodes * (size_t)kp.cap;
@@ -980,12 +1114,15 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
   w.exhausted = 0;
   w.cnt = 0;
   w.gather_calls = 0;
+  w.donate_tick = 0;
+  w.steal_fails = 0;
   w.wbytes = w.wmerge = w.wjobs = 0;
   if (lane == 0) {
     w.h->lock = 0;
     w.h->L = 0;
     w.h->root_it = 0;
     w.h->root_end = 0;
+    for (int i = 0; i <= STM_KMAX; ++i) w.h->lgen[i] = 1;
     for (int i = 0; i < STM_KMAX; ++i) {
       w.h->nsib[i] = 0;
       w.h->cur[i] = 0;
@@ -1096,20 +1233,39 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
   }
 }
 
-int stm_smem_bytes(int block_warps, int k, int n_nodes) {
-  return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes);
+int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
+  return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);
 }
 
-int stm_occupancy(int block_warps, int k, int n_nodes, int* blocks_per_sm) {
-  int smem = stm_smem_bytes(block_warps, k, n_nodes);
+int stm_occupancy(int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm) {
+  int smem = stm_smem_bytes(block_warps, k, n_nodes, ht_slots);
   cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
+  // The DFS stacks are the only shared-memory users: carve out just enough shared
+  // memory for the register-limited number of resident blocks and leave the rest
+  // of the unified 256 KB array to L1, which caches the binary-search probes.
+  cudaFuncAttributes fa;
+  e = cudaFuncGetAttributes(&fa, stm_count_kernel);
+  if (e != cudaSuccess) return (int)e;
+  const int threads = block_warps * 32;
+  const int regs_per_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
+  int want = std::min(65536 / std::max(1, regs_per_warp * block_warps), 64 / block_warps);
+  want = std::max(1, std::min(want, 32));
+  const double need = (double)want * (smem + 1024);
+  int pct = (int)std::ceil(100.0 * need / (228.0 * 1024.0));
+  pct = std::max(0, std::min(100, pct));
+  if (const char* cv = getenv("STM_CARVEOUT")) pct = atoi(cv);  // experiments: -1 = leave the driver default
+  if (pct >= 0) {
+    e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+    if (e != cudaSuccess) return (int)e;
+  }
+  (void)threads;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, stm_count_kernel, block_warps * 32, smem);
   return (int)e;
 }
 
 int stm_launch(const StmKParams& kp, int grid, void* stream) {
-  int smem = stm_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes);
+  int smem = stm_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes, kp.ht_slots);
   cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   void* args[] = {(void*)&kp};

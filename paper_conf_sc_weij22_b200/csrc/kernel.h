@@ -51,13 +51,16 @@ struct StmKParams {
   int32_t rank, world, chunk;
   int32_t local_steal, global_steal, stop_level, detect_level, unroll, root_batch;
   int32_t count_bytes;            // 1 = accumulate algorithmic bytes (instrumented launch)
+  int32_t ht_slots;               // per-warp shared-memory hash slots (0 = off)
+  int32_t donate_mask;            // donors look for idle blocks every (mask+1)-th opportunity
+  int32_t backoff_max;            // idle warps sleep up to 32 << backoff_max ns between steal attempts
   long long watchdog_cycles;      // debug: abort (set work->overflow = 2) after this many cycles; 0 = off
   uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
 };
 
 // size in bytes of the dynamic shared memory for one block
-int stm_smem_bytes(int block_warps, int k, int n_nodes);
+int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
 // launches the persistent kernel (cooperative); returns cudaError_t as int
 int stm_launch(const StmKParams& kp, int grid, void* stream);
 // max co-resident blocks per SM for the given block size
-int stm_occupancy(int block_warps, int k, int n_nodes, int* blocks_per_sm);
+int stm_occupancy(int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);

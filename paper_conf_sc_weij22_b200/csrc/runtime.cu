@@ -309,11 +309,18 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.detect_level = t.detect_level;
   kp.unroll = t.unroll;
   kp.root_batch = std::max(1, std::min(STM_RMAX, t.root_chunk));
-  kp.count_bytes = t.debug_per_root == 2 ? 1 : 0;  // reserved field doubles as the instrumentation switch
+  kp.count_bytes = t.instrument ? 1 : 0;
+  if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
+    return stm_fail(STM_EINVAL, "hash_slots %d: 0 or a power of two in 64..4096", t.hash_slots);
+  kp.ht_slots = t.hash_slots;
+  kp.donate_mask = 0;  // look for idle blocks at every opportunity (measured: rate limiting starves idle blocks)
+  kp.backoff_max = 8;
+  if (const char* x = getenv("STM_DONATE_MASK")) kp.donate_mask = atoi(x);  // experiments
+  if (const char* x = getenv("STM_BACKOFF_MAX")) kp.backoff_max = atoi(x);
   if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
 
   int bps = 0;
-  int oe = stm_occupancy(t.block_warps, P.k, P.n_nodes, &bps);
+  int oe = stm_occupancy(t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy: %s", cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -369,7 +376,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
   g_info.grid = grid;
   g_info.block_threads = t.block_warps * 32;
-  g_info.smem_bytes = stm_smem_bytes(t.block_warps, P.k, P.n_nodes);
+  g_info.smem_bytes = stm_smem_bytes(t.block_warps, P.k, P.n_nodes, t.hash_slots);
   g_info.arena_bytes = (int64_t)arena_bytes;
   g_info.cap = kp.cap;
   if (d_count_out) {

@@ -108,7 +108,7 @@ class MultiGPUCounter:
     def count_instrumented(self, plan: stm.Plan):
         """Untimed launch that also measures the algorithmic bytes."""
         t = stm.stm_tuning_default(**{f[0]: getattr(self.tuning, f[0]) for f in self.tuning._fields_})
-        t.debug_per_root = 2
+        t.instrument = 1
         if self.world == 1:
             c = stm.stm_match_count_ex(self.G.handle, plan.handle, t, None, None)
             return c, stm.stm_last_launch()

@@ -12,7 +12,7 @@ from typing import Optional, Sequence, Tuple
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libstm.so")
+LIB_PATH = os.environ.get("STM_LIB_PATH") or os.path.join(_HERE, "libstm.so")  # override: A/B experiments only
 
 STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW = range(6)
 STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
@@ -33,7 +33,7 @@ class StmError(RuntimeError):
 class stm_tuning(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("local_steal", "global_steal", "stop_level", "detect_level",
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
-                                               "debug_per_root")]
+                                               "instrument", "hash_slots")]
 
 
 class stm_shard(ctypes.Structure):

@@ -1,0 +1,29 @@
+"""Min-of-N timing of single queries through the C ABI: python tools/perf.py c2:k4,c2:c4,c5:k5 [key=val tuning...]"""
+import os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+os.environ.setdefault("STM_WATCHDOG_S", "60")
+import stmgen
+from paper_conf_sc_weij22_b200 import stm
+specs = sys.argv[1].split(",")
+tk = dict(a.split("=") for a in sys.argv[2:] if "=" in a)
+reps = int(tk.pop("reps", 3))
+graphs = {}
+for spec in specs:
+    cfg, name = spec.split(":")[:2]
+    vi = spec.endswith(":vi")
+    if cfg not in graphs:
+        g = stmgen.config_graph(cfg)
+        graphs[cfg] = (g, stm.Graph.from_stmgen(g))
+    g, G = graphs[cfg]
+    p = stmgen.CATALOG[name]
+    lab = stmgen.pattern_labels(p.k, 8, 7) if g.labels is not None else None
+    plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi)
+    t = stm.stm_tuning_default(**{k: int(v) for k, v in tk.items()})
+    best = 1e9
+    try:
+        for _ in range(reps):
+            t0 = time.perf_counter(); c = stm.count(G, plan, t); best = min(best, time.perf_counter() - t0)
+        info = stm.stm_last_launch()
+        print(f"{spec:16} {tk} count {c:>16} best {best*1e3:9.2f} ms  {c/best:.3e} m/s  ls={info['local_steals']} gs={info['global_steals']} grid={info['grid']} smem={info['smem_bytes']}", flush=True)
+    except Exception as e:
+        print(f"{spec:16} {tk} ERR {e}", flush=True)
