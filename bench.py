@@ -224,13 +224,15 @@ def main():
                                   cross_steal=not args.no_cross_steal)
 
     # ---- reference counts + algorithmic bytes (one instrumented, untimed launch per query)
-    counts, alg, merge, jobs = [], [], [], []
+    counts, alg, merge, jobs, idle, ranked = [], [], [], [], [], []
     for pl in plans:
         c, info = layer.count_instrumented(pl)
         counts.append(c)
         alg.append(info["alg_bytes"])
         merge.append(info["merge_bytes"])
         jobs.append(info["jobs"])
+        idle.append(info["idle_cycles"] / info["warp_cycles"] if info["warp_cycles"] else None)
+        ranked.append(bool(info["ranked"]))
 
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     d_counts = torch.zeros(len(plans), dtype=torch.int64, device=dev)
@@ -317,7 +319,8 @@ def main():
             tq = statistics.mean(launch_ms[qi]) / 1000.0
             per_q.append({"pattern": p, "mode": "vertex" if vi else "edge", "labels": lab, "count": counts[qi],
                           "query_time_s": round(tq, 6), "matches_per_s": counts[qi] / tq if tq else None,
-                          "alg_bytes": alg[qi], "merge_bytes": merge[qi], "set_ops": jobs[qi]})
+                          "alg_bytes": alg[qi], "merge_bytes": merge[qi], "set_ops": jobs[qi],
+                          "idle_steal_fraction": idle[qi], "degree_ranked": ranked[qi]})
         info = stm.stm_last_launch()
         line = {
             "metric": "query time (s) and matches/s per pattern×graph at 1/2/4/8 B200",

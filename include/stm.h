@@ -146,6 +146,11 @@ typedef struct stm_tuning {
   int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
   int32_t hash_slots;     /* per-warp shared-memory hash set for operands shared by a combined set
                              operation: 0 = off, else a power of two in 64..4096 slots. Default 0. */
+  int32_t vertex_order;   /* 0 = plans whose restrictions are order-free (STM_AUTO_RESTRICT, or none)
+                             count on the graph's degree-ranked copy: same count (any total order of V
+                             breaks the symmetry), far less work on skewed graphs; per-root output
+                             then attributes each match to f(order[0]) minimal in (degree, id) order.
+                             1 = always the caller's vertex ids.  Default 0. */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -218,6 +223,12 @@ typedef struct stm_launch_info {
   int64_t alg_bytes;       /* algorithmic bytes W; instrumented calls only (tuning.instrument == 1) */
   int64_t merge_bytes;     /* merge-equivalent bytes W_merge; instrumented calls only */
   int64_t jobs;            /* set operations executed; instrumented calls only */
+  int32_t ranked;          /* 1 = counted on the degree-ranked copy (stm_tuning.vertex_order) */
+  int32_t reserved;
+  int64_t idle_cycles;     /* sum over warps of SM cycles spent acquiring work (root cursor, stealing,
+                              waiting idle); instrumented calls only */
+  int64_t warp_cycles;     /* sum over warps of their lifetime in SM cycles; instrumented calls only.
+                              idle_cycles / warp_cycles = idle/stealing fraction of warps */
 } stm_launch_info;
 
 stm_status stm_last_launch(stm_launch_info* info);

@@ -256,6 +256,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   P->restr = R;
   P->aut = aut;
   P->flags = flags;
+  P->order_free = (flags & STM_AUTO_RESTRICT) || R.empty();
   StmPlan& D = P->dev;
   memset(&D, 0, sizeof D);
   D.k = k;
@@ -284,6 +285,24 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
       if (less[pi[l]][pi[j]]) hi_pos[l] |= 1u << j;
       if (!adj[pi[l]][pi[j]]) excl[l] |= 1u << j;
     }
+
+  // Drop dominated bounds: w > v_j is implied by w > v_j' when f(pi[j]) < f(pi[j'])
+  // already holds (transitive closure), so only the maximal lower and minimal upper
+  // bound positions are kept (one compare each for cliques instead of up to k-1).
+  auto reduce_lo = [&](unsigned m) {
+    unsigned r = m;
+    for (int j = 0; j < k; ++j)
+      for (int j2 = 0; j2 < k; ++j2)
+        if ((m >> j & 1) && (m >> j2 & 1) && j != j2 && less[pi[j]][pi[j2]]) r &= ~(1u << j);
+    return r;
+  };
+  auto reduce_hi = [&](unsigned m) {
+    unsigned r = m;
+    for (int j = 0; j < k; ++j)
+      for (int j2 = 0; j2 < k; ++j2)
+        if ((m >> j & 1) && (m >> j2 & 1) && j != j2 && less[pi[j2]][pi[j]]) r &= ~(1u << j);
+    return r;
+  };
 
   // ---- operation chains and the code-motion trie
   struct TNode {
@@ -383,8 +402,8 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     }
     unsigned known = (1u << x.level) - 1;  // v_0..v_{level-1}
     n.lab = (uint8_t)lm;
-    n.lo = (uint8_t)(lo & known);
-    n.hi = (uint8_t)(hi & known);
+    n.lo = (uint8_t)reduce_lo(lo & known);
+    n.hi = (uint8_t)reduce_hi(hi & known);
   }
   for (int l = 0; l <= k; ++l) D.level_begin[l] = 0;
   for (int l = 0; l < k; ++l) {
@@ -405,8 +424,8 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   if (D.cnt_a.kind == STM_SRC_NODE) D.cnt_a.idx = (int8_t)remap[D.cnt_a.idx];
   for (int l = 0; l < k; ++l) {
     D.filt[l].lab = (uint8_t)labmask(l);
-    D.filt[l].lo = (uint8_t)lo_pos[l];
-    D.filt[l].hi = (uint8_t)hi_pos[l];
+    D.filt[l].lo = (uint8_t)reduce_lo(lo_pos[l]);
+    D.filt[l].hi = (uint8_t)reduce_hi(hi_pos[l]);
     D.filt[l].excl = (uint8_t)excl[l];
   }
   build_describe(P);

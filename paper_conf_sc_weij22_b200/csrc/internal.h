@@ -17,6 +17,7 @@ struct stm_plan {
   std::vector<std::pair<int, int>> restr;
   int64_t aut = 0;
   uint32_t flags = 0;
+  bool order_free = false;  // restrictions hold for every total order of V (GK or none)
   std::string describe;
 };
 

@@ -80,6 +80,7 @@ struct W {
   unsigned donate_tick;
   int steal_fails;
   unsigned long long wbytes, wmerge, wjobs;  // per-lane instrumentation partials
+  unsigned long long idle_cyc;               // cycles in acquire_work (instrumented launches)
   int* ht;                          // shared-memory hash set (HT_SLOTS ints)
   unsigned ht_mask;
   unsigned long long ht_ptr;        // key of the hashed operand
@@ -142,10 +143,8 @@ __device__ __forceinline__ void bounds(const W& w, unsigned lo_m, unsigned hi_m,
                                        int& lo, int& hi) {
   lo = -1;
   hi = INT_MAX;
-  for (int j = 0; j < STM_KMAX; ++j) {
-    if (lo_m & (1u << j)) lo = max(lo, pval(w, j, F, u, c));
-    if (hi_m & (1u << j)) hi = min(hi, pval(w, j, F, u, c));
-  }
+  for (unsigned m = lo_m; m; m &= m - 1) lo = max(lo, pval(w, __ffs(m) - 1, F, u, c));
+  for (unsigned m = hi_m; m; m &= m - 1) hi = min(hi, pval(w, __ffs(m) - 1, F, u, c));
 }
 
 __device__ __forceinline__ bool labok(const W& w, int x, unsigned lab) {
@@ -379,7 +378,10 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
       jc -= 1;
     }
   }
-  if (w.kp->per_root && mine && jc) atomicAdd(&w.kp->per_root[pval(w, 0, F, J.u, J.c)], jc);
+  if (w.kp->per_root && mine && jc) {
+    const int r = pval(w, 0, F, J.u, J.c);
+    atomicAdd(&w.kp->per_root[w.kp->root_map ? w.kp->root_map[r] : r], jc);
+  }
   unsigned long long s = jc;
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(FULLMASK, s, o);
@@ -1117,6 +1119,7 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
   w.donate_tick = 0;
   w.steal_fails = 0;
   w.wbytes = w.wmerge = w.wjobs = 0;
+  w.idle_cyc = 0;
   if (lane == 0) {
     w.h->lock = 0;
     w.h->L = 0;
@@ -1161,7 +1164,12 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
       }
       if (lk) unlock_ws(w, w.h);
       if (m == 0) {
-        if (!acquire_work(w, t0)) break;
+        // instrumented launches: time spent acquiring work (cursor, stealing, idle
+        // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
+        const long long ta = kp.count_bytes ? clock64() : 0;
+        const bool got = acquire_work(w, t0);
+        if (kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
+        if (!got) break;
       }
       continue;
     }
@@ -1226,6 +1234,8 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
       w.wjobs += __shfl_xor_sync(FULLMASK, w.wjobs, o);
     }
     if (lane == 0) {
+      atomicAdd(&kp.work->idle_cycles, w.idle_cyc);
+      atomicAdd(&kp.work->warp_cycles, (unsigned long long)(clock64() - t0));
       atomicAdd(&kp.work->alg_bytes, w.wbytes);
       atomicAdd(&kp.work->merge_bytes, w.wmerge);
       atomicAdd(&kp.work->n_jobs, w.wjobs);

@@ -26,6 +26,8 @@ struct StmWork {
   unsigned long long alg_bytes;    // SURVEY.md 8(d) W = sum W_op (instrumented launches only)
   unsigned long long merge_bytes;  // W_merge = sum 4(|A|+|B|)
   unsigned long long n_jobs;
+  unsigned long long idle_cycles;  // sum over warps of cycles spent acquiring work (instrumented)
+  unsigned long long warp_cycles;  // sum over warps of their lifetime in cycles (instrumented)
 };
 
 struct StmBlockSlot {             // per block, global memory (Fig. 6)
@@ -46,7 +48,8 @@ struct StmKParams {
   int32_t* arena;                 // [total_warps][n_nodes][cap]
   StmWork* work;
   StmBlockSlot* slots;            // [gridDim.x]
-  unsigned long long* per_root;   // [n] or NULL
+  unsigned long long* per_root;   // [n] or NULL (indexed by the caller's vertex id)
+  const int32_t* root_map;        // counting id -> caller's id (degree-ranked copy), or NULL
   unsigned long long* cursors[8]; // chunk cursors (own rank + optional peers)
   int32_t rank, world, chunk;
   int32_t local_steal, global_steal, stop_level, detect_level, unroll, root_batch;

@@ -11,6 +11,9 @@
 #include <thread>
 #include <vector>
 
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
 #include <cuda_runtime.h>
 
 #include "internal.h"
@@ -66,6 +69,15 @@ struct stm_graph {
   bool owns_csr = true;
   std::vector<int32_t> label_values;  // dense id -> label value
   int num_sms = 0;
+  // Degree-ranked copy: vertex i of
+  // the copy is the i-th vertex in (degree, id) order.  Plans whose restrictions
+  // are order-free (STM_AUTO_RESTRICT or none) count on it; the count is the same
+  // (any total order breaks symmetry), the work far smaller on skewed graphs.
+  bool ranked = false;
+  int64_t* d_rrow_ptr = nullptr;
+  int32_t* d_rcol_idx = nullptr;
+  uint8_t* d_rlabels = nullptr;
+  int32_t* d_rank2orig = nullptr;  // [n]: ranked id -> caller's id (per-root output)
   std::mutex mu;
   std::map<void*, Scratch> scratch;  // per stream
 };
@@ -78,6 +90,96 @@ __global__ void degree_scan(const int64_t* rp, int64_t n, long long* out) {
     if (d < 0) out[1] = 1;
     else atomicMax(&out[0], d);
   }
+}
+
+// ---------------------------------------------------------------- degree-ranked copy
+__global__ void rank_keys(const int64_t* rp, int64_t n, unsigned long long* keys) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    keys[v] = ((unsigned long long)(rp[v + 1] - rp[v]) << 32) | (unsigned long long)v;
+}
+__global__ void rank_scatter(const unsigned long long* sorted, int64_t n, int32_t* rank2orig, int32_t* orig2rank,
+                             int64_t* newdeg, const uint8_t* lab, uint8_t* rlab) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = (int32_t)(sorted[i] & 0xffffffffull);
+    rank2orig[i] = v;
+    orig2rank[v] = (int32_t)i;
+    newdeg[i] = (int64_t)(sorted[i] >> 32);
+    if (lab) rlab[i] = lab[v];
+  }
+}
+// one warp per ranked row: the caller's row of rank2orig[i], renumbered (unsorted)
+__global__ void rank_fill(const int64_t* rp, const int32_t* ci, const int32_t* rank2orig, const int32_t* orig2rank,
+                          const int64_t* rrp, int32_t* out, int64_t n) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < n;
+       i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const int32_t v = rank2orig[i];
+    const int64_t b = rp[v], d = rp[v + 1] - b, o = rrp[i];
+    for (int64_t j = lane; j < d; j += 32) out[o + j] = orig2rank[ci[b + j]];
+  }
+}
+
+// Builds g's degree-ranked copy on the device (load time, not the query).  Only
+// speed depends on it: when it cannot be built (sizes beyond CUB's int range, no
+// memory) `ranked` stays false and every plan counts on the caller's numbering.
+static void build_ranked(stm_graph* g) {
+  const int64_t n = g->n, nnz = g->nnz;
+  if (n < 2 || nnz < 1 || nnz > INT32_MAX) return;
+  unsigned long long *keys = nullptr, *skeys = nullptr;
+  int32_t* orig2rank = nullptr;
+  int32_t* tmpcol = nullptr;
+  void* temp = nullptr;
+  size_t t1 = 0, t2 = 0, t3 = 0;
+  cudaError_t e = cudaSuccess;
+  auto ok = [&](cudaError_t x) { if (e == cudaSuccess) e = x; return e == cudaSuccess; };
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 8 * 1024);
+  ok(cudaMalloc(&keys, sizeof(unsigned long long) * n));
+  ok(cudaMalloc(&skeys, sizeof(unsigned long long) * n));
+  ok(cudaMalloc(&orig2rank, sizeof(int32_t) * n));
+  ok(cudaMalloc(&g->d_rank2orig, sizeof(int32_t) * n));
+  ok(cudaMalloc(&g->d_rrow_ptr, sizeof(int64_t) * (n + 1)));
+  ok(cudaMalloc(&g->d_rcol_idx, sizeof(int32_t) * nnz));
+  ok(cudaMalloc(&tmpcol, sizeof(int32_t) * nnz));
+  if (g->d_labels) ok(cudaMalloc(&g->d_rlabels, n));
+  if (e == cudaSuccess) {
+    int end_bit = 33;
+    while (end_bit < 64 && (g->max_degree >> (end_bit - 32)) != 0) ++end_bit;
+    ok(cub::DeviceRadixSort::SortKeys(nullptr, t1, keys, skeys, (int)n, 0, end_bit));
+    ok(cub::DeviceScan::ExclusiveSum(nullptr, t2, g->d_rrow_ptr, g->d_rrow_ptr, (int)(n + 1)));
+    ok(cub::DeviceSegmentedSort::SortKeys(nullptr, t3, tmpcol, g->d_rcol_idx, (int)nnz, (int)n, g->d_rrow_ptr,
+                                          g->d_rrow_ptr + 1));
+    ok(cudaMalloc(&temp, std::max<size_t>(std::max(t1, std::max(t2, t3)), 16)));
+    if (e == cudaSuccess) {
+      rank_keys<<<grid, 256>>>(g->d_row_ptr, n, keys);
+      ok(cub::DeviceRadixSort::SortKeys(temp, t1, keys, skeys, (int)n, 0, end_bit));
+      ok(cudaMemset(g->d_rrow_ptr + n, 0, sizeof(int64_t)));
+      rank_scatter<<<grid, 256>>>(skeys, n, g->d_rank2orig, orig2rank, g->d_rrow_ptr, g->d_labels, g->d_rlabels);
+      ok(cub::DeviceScan::ExclusiveSum(temp, t2, g->d_rrow_ptr, g->d_rrow_ptr, (int)(n + 1)));
+      rank_fill<<<grid, 256>>>(g->d_row_ptr, g->d_col_idx, g->d_rank2orig, orig2rank, g->d_rrow_ptr, tmpcol, n);
+      ok(cub::DeviceSegmentedSort::SortKeys(temp, t3, tmpcol, g->d_rcol_idx, (int)nnz, (int)n, g->d_rrow_ptr,
+                                            g->d_rrow_ptr + 1));
+      ok(cudaGetLastError());
+      ok(cudaDeviceSynchronize());
+    }
+  }
+  cudaFree(keys);
+  cudaFree(skeys);
+  cudaFree(orig2rank);
+  cudaFree(tmpcol);
+  cudaFree(temp);
+  if (e == cudaSuccess) {
+    g->ranked = true;
+    return;
+  }
+  cudaGetLastError();  // clear the non-sticky error (e.g. out of memory)
+  cudaFree(g->d_rank2orig);
+  cudaFree(g->d_rrow_ptr);
+  cudaFree(g->d_rcol_idx);
+  cudaFree(g->d_rlabels);
+  g->d_rank2orig = nullptr;
+  g->d_rrow_ptr = nullptr;
+  g->d_rcol_idx = nullptr;
+  g->d_rlabels = nullptr;
 }
 
 static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci) {
@@ -166,6 +268,7 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
                     cudaGetErrorString(e));
   }
+  build_ranked(g);
   *out = g;
   return STM_OK;
 }
@@ -221,6 +324,7 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
     }
   }
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  build_ranked(g);
   *out = g;
   return STM_OK;
 }
@@ -245,6 +349,10 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
     cudaFree(g->d_col_idx);
   }
   cudaFree(g->d_labels);
+  cudaFree(g->d_rank2orig);
+  cudaFree(g->d_rrow_ptr);
+  cudaFree(g->d_rcol_idx);
+  cudaFree(g->d_rlabels);
   delete g;
   return STM_OK;
 }
@@ -291,9 +399,12 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   StmKParams kp;
   memset(&kp, 0, sizeof kp);
   kp.plan = P;
-  kp.row_ptr = g->d_row_ptr;
-  kp.col_idx = g->d_col_idx;
-  kp.labels = g->d_labels;
+  // order-free restrictions count on the degree-ranked copy (same count, less work)
+  const bool use_rank = g->ranked && p->order_free && t.vertex_order == 0;
+  kp.row_ptr = use_rank ? g->d_rrow_ptr : g->d_row_ptr;
+  kp.col_idx = use_rank ? g->d_rcol_idx : g->d_col_idx;
+  kp.labels = use_rank ? g->d_rlabels : g->d_labels;
+  kp.root_map = use_rank ? g->d_rank2orig : nullptr;
   kp.n = g->n;
   // label-slot table: dense graph label -> bitmask of pattern slots with that value
   for (int d = 0; d < (int)g->label_values.size(); ++d)
@@ -379,6 +490,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   g_info.smem_bytes = stm_smem_bytes(t.block_warps, P.k, P.n_nodes, t.hash_slots);
   g_info.arena_bytes = (int64_t)arena_bytes;
   g_info.cap = kp.cap;
+  g_info.ranked = use_rank ? 1 : 0;
   if (d_count_out) {
     CU(cudaMemcpyAsync(d_count_out, &work->count, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
   }
@@ -394,6 +506,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     g_info.alg_bytes = (int64_t)hw.alg_bytes;
     g_info.merge_bytes = (int64_t)hw.merge_bytes;
     g_info.jobs = (int64_t)hw.n_jobs;
+    g_info.idle_cycles = (int64_t)hw.idle_cycles;
+    g_info.warp_cycles = (int64_t)hw.warp_cycles;
     *h_count = hw.count;
   }
   return STM_OK;

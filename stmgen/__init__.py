@@ -188,6 +188,19 @@ def relabel(g: Graph, perm_seed: int) -> Graph:
     return out
 
 
+def permute(g: Graph, p: np.ndarray) -> Graph:
+    """Same graph with vertex v renamed p[v] (labels carried along)."""
+    src = np.repeat(np.arange(g.n, dtype=np.int64), np.diff(g.row_ptr))
+    e = np.stack([src, g.col_idx.astype(np.int64)], 1)
+    p = np.asarray(p, dtype=np.int64)
+    out = from_edges(g.n, p[e], name=g.name + "_permuted")
+    if g.labels is not None:
+        lab = np.empty(g.n, np.int32)
+        lab[p] = g.labels
+        out.labels = lab
+    return out
+
+
 def empty(n: int) -> Graph:
     return from_edges(n, np.zeros((0, 2), np.int64), name=f"empty{n}")
 

@@ -119,6 +119,7 @@ TUNINGS = [
     dict(unroll=1), dict(unroll=2), dict(unroll=16),
     dict(root_chunk=1, stop_level=3, detect_level=3),
     dict(block_warps=4), dict(block_warps=32, blocks_per_sm=1),
+    dict(vertex_order=1), dict(vertex_order=1, unroll=1, local_steal=0, global_steal=0),
 ]
 
 
@@ -177,15 +178,35 @@ def test_config_scale_sampled_roots(cfg, name, ntop):
     G = stm.Graph.from_stmgen(g)
     p = CATALOG[name]
     plan = stm.Plan(p.k, p.edges)
-    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
-    assert int(pr.sum(dtype=np.uint64)) == tot
+    R = oracle.gk_restrictions(p.k, p.edges)
     rng = np.random.default_rng(5)
     deg = g.degrees()
+    # caller's numbering (vertex_order=1)
+    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(vertex_order=1))
+    assert int(pr.sum(dtype=np.uint64)) == tot
     top = np.argsort(deg)[len(deg) - ntop:] if ntop else np.zeros(0, np.int64)
     roots = np.unique(np.concatenate([rng.choice(g.n, 48, replace=False), top]))
-    R = oracle.gk_restrictions(p.k, p.edges)
     oc, opr = oracle.count(g, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=roots, per_root=True)
     assert np.array_equal(pr[roots], opr)
+    # default: degree-ranked symmetry breaking, as bench.py times it; the oracle runs on
+    # the graph renumbered in (degree, id) order
+    tot2, pr2 = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
+    assert stm.stm_last_launch()["ranked"] == 1
+    assert tot2 == tot and int(pr2.sum(dtype=np.uint64)) == tot
+    rank2orig, gr = degree_ranked(g)
+    rroots = np.unique(np.concatenate([rng.choice(g.n, 48, replace=False), np.arange(g.n - ntop, g.n)]))
+    oc2, opr2 = oracle.count(gr, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=rroots,
+                             per_root=True)
+    assert np.array_equal(pr2[rank2orig[rroots]], opr2)
+
+
+def degree_ranked(g):
+    """(rank2orig, g renumbered so that vertex i is the i-th in (degree, id) order)."""
+    deg = g.degrees()
+    rank2orig = np.lexsort((np.arange(g.n), deg))
+    perm = np.empty(g.n, np.int64)
+    perm[rank2orig] = np.arange(g.n)
+    return rank2orig, stmgen.permute(g, perm)
 
 
 def test_degenerate_graphs():
@@ -203,9 +224,17 @@ def test_per_root_histogram(rmat_small):
     for name, vi in [("diamond", False), ("house", True), ("k4", False)]:
         p = CATALOG[name]
         plan = stm.Plan(p.k, p.edges, vertex_induced=vi)
-        tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(root_chunk=1))
         R = oracle.gk_restrictions(p.k, p.edges)
+        tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle,
+                                               stm.stm_tuning_default(root_chunk=1, vertex_order=1))
         otot, opr = oracle.count(g, p.k, p.edges, vertex_induced=vi, restrictions=R,
                                  root_u=plan.first_vertex, per_root=True)
         assert tot == otot
         assert np.array_equal(pr, opr)
+        # degree-ranked (default): attribution to the (degree, id)-minimal root
+        tot2, pr2 = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(root_chunk=1))
+        rank2orig, gr = degree_ranked(g)
+        otot2, opr2 = oracle.count(gr, p.k, p.edges, vertex_induced=vi, restrictions=R,
+                                   root_u=plan.first_vertex, per_root=True)
+        assert tot2 == otot2 == otot
+        assert np.array_equal(pr2[rank2orig], opr2)

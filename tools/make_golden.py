@@ -29,6 +29,14 @@ CASES = [
     ("c4_k4_L_ei", "c4", "k4", False, (0, 1, 2, 3)),
     ("c3_k5_ei", "c3", "k5", False, None),
     ("c4_diamond_L_ei", "c4", "diamond", False, (0, 1, 1, 2)),
+    ("c2_c4_ei", "c2", "c4", False, None),
+    ("c4_k6me_L_ei", "c4", "k6_minus_e", False, (0, 1, 2, 3, 4, 5)),
+    ("c4_w5_L_ei", "c4", "w5", False, (0, 1, 1, 2, 2, 3)),
+    ("c4_c6_L_vi", "c4", "c6", True, (0, 1, 2, 0, 1, 2)),
+    ("c4_w6_L_ei", "c4", "w6", False, (0, 1, 2, 1, 2, 1, 2)),
+    ("c4_c7_L_vi", "c4", "c7", True, (0, 1, 2, 3, 0, 1, 2)),
+    ("c3_house_ei", "c3", "house", False, None),
+    ("c3_c5_ei", "c3", "c5", False, None),
 ]
 
 
