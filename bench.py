@@ -38,8 +38,8 @@ import numpy as np  # noqa: E402
 
 WORKLOADS = {
     # name: (config graph, [(pattern, vertex_induced, labels)], description)
-    "c5": ("c5", [("k5", False, None), ("prism", False, None)],
-           "configs[4]: 5-clique + prism (size 6) on LiveJournal-shaped R-MAT s23 (5.45M v, 46M e)"),
+    "c5": ("c5", [("k5", False, None), ("k6_minus_e", False, None)],
+           "configs[4]: 5-clique + K6-e (size 6) on LiveJournal-shaped R-MAT s23 (5.45M v, 46M e)"),
     "c2": ("c2", [("k4", False, None), ("c4", False, None)],
            "configs[1]: 4-clique + 4-cycle on R-MAT s16 (65k v, 0.9M e)"),
     "c3": ("c3", [("k5", False, None), ("house", False, None), ("c5", False, None)],
@@ -48,6 +48,10 @@ WORKLOADS = {
            "configs[3]: labeled size-6 patterns (8 labels) on MiCo-shaped R-MAT s17"),
     "c1": ("c1", [("triangle", False, None)], "configs[0]: triangles on ER(1000, 10k)"),
 }
+
+
+def log(msg):
+    print(f"[bench] {msg}", file=sys.stderr, flush=True)
 
 
 def env_int(name, default):
@@ -213,8 +217,11 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     cfg, queries, desc = WORKLOADS[args.workload]
+    t_start = time.time()
     g = stmgen.config_graph(cfg)
+    log(f"graph {cfg} generated in {time.time() - t_start:.1f}s (n={g.n}, nnz={g.row_ptr[-1]})")
     G = stm.Graph.from_stmgen(g, device=local)
+    log(f"graph loaded ({time.time() - t_start:.1f}s)")
     plans = [stm.Plan(stmgen.CATALOG[p].k, stmgen.CATALOG[p].edges, lab, vertex_induced=vi)
              for p, vi, lab in queries]
     stream = torch.cuda.current_stream(dev)
@@ -234,6 +241,7 @@ def main():
         idle.append(info["idle_cycles"] / info["warp_cycles"] if info["warp_cycles"] else None)
         ranked.append(bool(info["ranked"]))
 
+    log(f"instrumented launches done ({time.time() - t_start:.1f}s): counts {counts}")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     d_counts = torch.zeros(len(plans), dtype=torch.int64, device=dev)
 
@@ -309,6 +317,7 @@ def main():
         e2e["value"] = matches_per_step / e2e.pop("seconds_per_step")
         e2e["unit"] = "matches/s"
 
+    log(f"timed + e2e done ({time.time() - t_start:.1f}s)")
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = oracle_sample(g, queries, plans, budget_s=args.cpu_budget)

@@ -145,7 +145,8 @@ typedef struct stm_tuning {
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
   int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
   int32_t hash_slots;     /* per-warp shared-memory hash set for operands shared by a combined set
-                             operation: 0 = off, else a power of two in 64..4096 slots. Default 0. */
+                             operation: 0 = off, else a power of two in 64..4096 slots. Default 0.
+                             Only in builds with -DSTM_WITH_HASH=1 (else STM_EUNSUPPORTED): measured slower. */
   int32_t vertex_order;   /* 0 = plans whose restrictions are order-free (STM_AUTO_RESTRICT, or none)
                              count on the graph's degree-ranked copy: same count (any total order of V
                              breaks the symmetry), far less work on skewed graphs; per-root output

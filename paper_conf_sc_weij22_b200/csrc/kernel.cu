@@ -36,6 +36,9 @@
 #include "kernel.h"
 
 #define FULLMASK 0xffffffffu
+#ifndef STM_WITH_HASH
+#define STM_WITH_HASH 0  // per-warp shared-memory hash sets (stm_tuning.hash_slots): measured slower, off
+#endif
 #define HT_MIN 16
 
 namespace {
@@ -94,19 +97,28 @@ struct W {
 
 __device__ __forceinline__ int bcast(int x) { return __shfl_sync(FULLMASK, x, 0); }
 
+// Branchless binary searches (a select per probe, ceil(log2 n) dependent loads):
+// lbound = #elements < x; member = x in a.  Lanes with equal n stay converged.
 __device__ __forceinline__ int lbound(const int* __restrict__ a, int n, int x) {
-  int lo = 0;
-  while (n > 0) {
-    int half = n >> 1;
-    int v = a[lo + half];
-    if (v < x) { lo += half + 1; n -= half + 1; } else { n = half; }
+  if (n <= 0) return 0;
+  const int* base = a;
+  while (n > 1) {
+    const int half = n >> 1;
+    base = (base[half] < x) ? base + half : base;
+    n -= half;
   }
-  return lo;
+  return (int)(base - a) + (*base < x);
 }
 
-__device__ __forceinline__ bool member(const int* a, int n, int x) {
-  int p = lbound(a, n, x);
-  return p < n && a[p] == x;
+__device__ __forceinline__ bool member(const int* __restrict__ a, int n, int x) {
+  if (n <= 0) return false;
+  const int* base = a;
+  while (n > 1) {
+    const int half = n >> 1;
+    base = (base[half] <= x) ? base + half : base;
+    n -= half;
+  }
+  return *base == x;
 }
 
 __device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) {
@@ -240,9 +252,9 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
   int hn = 0;
   int hnode = 0;
   const int ht_max = w.kp->ht_slots / 2;
-  if (sameA && al0 >= HT_MIN && al0 <= ht_max && b0 != 0ull) {  // (warp-uniform: lane 0 owns a job)
+  if (STM_WITH_HASH && sameA && al0 >= HT_MIN && al0 <= ht_max && b0 != 0ull) {  // (warp-uniform: lane 0 owns a job)
     hmode = 1; hp = (const int*)a0; hn = al0; hnode = __shfl_sync(FULLMASK, J.a_node, 0);
-  } else if (sameB && bl0 >= HT_MIN && bl0 <= ht_max) {
+  } else if (STM_WITH_HASH && sameB && bl0 >= HT_MIN && bl0 <= ht_max) {
     hmode = 2; hp = (const int*)b0; hn = bl0;
   }
   if (hmode) {
@@ -333,7 +345,7 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
       x = Dj[e - sj];
       keep = x > loj && x < hij;
       if (keep && (fj & 1)) {
-        const bool f = (fj & 2) ? ht_has(ht, htmask, x) : member(Pj, pl, x);
+        const bool f = (STM_WITH_HASH && (fj & 2)) ? ht_has(ht, htmask, x) : member(Pj, pl, x);
         keep = (fj & 4) ? !f : f;
       }
       if (keep && labj != STM_LAB_ANY) keep = (l2s[glabels[x]] & labj) != 0;
@@ -1242,6 +1254,8 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
     }
   }
 }
+
+int stm_hash_compiled() { return STM_WITH_HASH; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
   return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);

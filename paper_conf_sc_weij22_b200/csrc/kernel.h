@@ -61,6 +61,8 @@ struct StmKParams {
   uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
 };
 
+// 1 if the shared-memory hash-set path is compiled in (-DSTM_WITH_HASH=1)
+int stm_hash_compiled();
 // size in bytes of the dynamic shared memory for one block
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
 // launches the persistent kernel (cooperative); returns cudaError_t as int

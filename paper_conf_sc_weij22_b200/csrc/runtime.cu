@@ -423,6 +423,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
     return stm_fail(STM_EINVAL, "hash_slots %d: 0 or a power of two in 64..4096", t.hash_slots);
+  if (t.hash_slots && !stm_hash_compiled())
+    return stm_fail(STM_EUNSUPPORTED, "hash_slots: this build has no hash-set path (-DSTM_WITH_HASH=1)");
   kp.ht_slots = t.hash_slots;
   kp.donate_mask = 0;  // look for idle blocks at every opportunity (measured: rate limiting starves idle blocks)
   kp.backoff_max = 8;
