@@ -140,7 +140,7 @@ typedef struct stm_tuning {
   int32_t stop_level;     /* frames < stop_level are stealable (paper: 2). Default 2. */
   int32_t detect_level;   /* donors look for idle blocks at frames < detect_level (paper: 1). Default 2. */
   int32_t unroll;         /* sibling iterations expanded together, 1..16 (paper: 8). Default 8. */
-  int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 32. */
+  int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 2 (measured best on B200). */
   int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
   int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
@@ -233,6 +233,18 @@ typedef struct stm_launch_info {
 } stm_launch_info;
 
 stm_status stm_last_launch(stm_launch_info* info);
+
+/*
+ * stm_last_profile -- per-phase cycle buckets of this thread's last synchronous call,
+ * filled only by libraries built with -DSTM_PROFILE=1 (A/B builds; zeros otherwise).
+ * out receives min(n, 40) uint64: for phase i in 0..11 (root gather, root sibling
+ * set-up, candidate gather, set-node build, frame count, fused count, donate,
+ * work acquisition, next-sibling set-up, descend set-up, combined-operation set-up,
+ * combined-operation element loop) the triple (warp cycles, calls, items), then
+ * the summed and the maximal warp lifetime, the summed and the maximal time (from
+ * the warp's start) at which the root cursors were first seen exhausted.
+ */
+stm_status stm_last_profile(uint64_t* out, int n);
 
 /* stm_last_error -- thread-local message for the last non-OK status of this thread. */
 const char* stm_last_error(void);

@@ -36,6 +36,41 @@
 #include "kernel.h"
 
 #define FULLMASK 0xffffffffu
+// A/B build switches (tools/gpu_variants.sh); the defaults are the measured best.
+#ifndef STM_JOBS_INLINE
+#define STM_JOBS_INLINE 1   // 0: one out-of-line copy of run_jobs (smaller code, W in local memory)
+#endif
+#ifndef STM_MAXT
+#define STM_MAXT 1024       // __launch_bounds__ max threads: 1024 -> 64 registers, 512 -> 128
+#endif
+#ifndef STM_STEP_NOINLINE
+#define STM_STEP_NOINLINE 0 // 1: build_nodes / gather_batch / fused_count out of line
+#endif
+#if STM_JOBS_INLINE
+#define JOBS_INL __forceinline__
+#else
+#define JOBS_INL __noinline__
+#endif
+#if STM_STEP_NOINLINE
+#define STEP_INL __noinline__
+#else
+#define STEP_INL
+#endif
+#ifndef STM_PROFILE
+#define STM_PROFILE 0       // 1: per-phase clock64() buckets (stm_last_profile); A/B builds only
+#endif
+#if STM_PROFILE
+#define PROF_BEGIN(id) const long long prof_t##id = clock64();
+#define PROF_END(id, items)                                    \
+  if (w.lane == 0) {                                           \
+    w.prof_cyc[id] += (unsigned long long)(clock64() - prof_t##id); \
+    w.prof_cnt[id] += 1;                                       \
+    w.prof_items[id] += (unsigned long long)(items);           \
+  }
+#else
+#define PROF_BEGIN(id)
+#define PROF_END(id, items)
+#endif
 #ifndef STM_WITH_HASH
 #define STM_WITH_HASH 0  // per-warp shared-memory hash sets (stm_tuning.hash_slots): measured slower, off
 #endif
@@ -84,6 +119,10 @@ struct W {
   int steal_fails;
   unsigned long long wbytes, wmerge, wjobs;  // per-lane instrumentation partials
   unsigned long long idle_cyc;               // cycles in acquire_work (instrumented launches)
+#if STM_PROFILE
+  unsigned long long prof_cyc[STM_PROF_N], prof_cnt[STM_PROF_N], prof_items[STM_PROF_N];
+  long long first_dry;  // clock64() when the root cursors were first seen exhausted
+#endif
   int* ht;                          // shared-memory hash set (HT_SLOTS ints)
   unsigned ht_mask;
   unsigned long long ht_ptr;        // key of the hashed operand
@@ -227,9 +266,10 @@ __device__ __forceinline__ int log2c(int n) { return 32 - __clz(n); }  // ceil(l
 
 // Returns the (warp-uniform) number of kept elements summed over all jobs when
 // counting; in materialise mode *outc (lane j) receives job j's output size.
-__device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F,
+__device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F,
                                                     unsigned excl, int* outc_lane) {
   const int lane = w.lane;
+  PROF_BEGIN(10)
   const bool mine = lane < njobs;
   // operands narrowed to the open interval (lo, hi) of the restriction bounds
   const int* An = J.A;
@@ -305,6 +345,8 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
     w.wmerge += 4ull * (unsigned long long)(an + bn);
     w.wjobs += 1;
   }
+  PROF_END(10, njobs)
+  PROF_BEGIN(11)
   int incl = dlen;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
@@ -369,6 +411,7 @@ __device__ unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, 
       outc += __popc(km & rmask);
     }
   }
+  PROF_END(11, total)
   if (!count_mode) {
     if (w.kp->count_bytes && mine) w.wbytes += 4ull * (unsigned long long)outc;
     *outc_lane = outc;
@@ -452,12 +495,27 @@ __device__ __forceinline__ int src_len(const W& w, int F, int u) {
   return len;
 }
 
+// Make sibling u current in frame F.  Its candidate list is sorted, so the level's
+// restriction bounds (lo, hi) select a contiguous position range: find it by
+// binary search instead of filtering every element (with degree-ranked ids a
+// hub's row is long but only its short suffix above v0 is a candidate).
+// Positions stay positions of the full list, so stolen ranges mean the same.
 __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
-  int len = src_len(w, F, u);
+  const int* p;
+  int len;
+  src_slice(w, w.P->cand[F], F, u, 0, 0, p, len);
+  const StmFilter f = w.P->filt[F];
+  int b = 0, e = len;
+  if ((f.lo | f.hi) && len > 0) {
+    int lo, hi;
+    bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
+    if (lo >= 0) b = lbound(p, len, lo + 1);
+    if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
+  }
   if (w.lane == 0) {
     w.h->cur[F] = u;
-    w.h->it[F] = 0;
-    w.h->end[F] = len;
+    w.h->it[F] = b;
+    w.h->end[F] = e;
   }
   __syncwarp();
 }
@@ -492,7 +550,7 @@ __device__ int node_ub(const W& w, int s, int F, int u, int c) {
 
 // Compute the nodes of level F+1 for the m siblings SIB(F+1, 0..m-1); offsets
 // NOFF were assigned by the caller; sizes NSZ are written here.
-__device__ void build_nodes(W& w, int F, int m) {
+__device__ STEP_INL void build_nodes(W& w, int F, int m) {
   const StmPlan& P = *w.P;
   const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
   if (nb == ne) return;
@@ -541,7 +599,7 @@ __device__ void build_nodes(W& w, int F, int m) {
 // siblings of frame F+1, admitted so that every node region fits.
 // Caller holds the frame lock if the frame is stealable.  Returns batch size.
 // ----------------------------------------------------------------------------
-__device__ int gather_batch(W& w, int F, int U) {
+__device__ STEP_INL int gather_batch(W& w, int F, int U) {
   const StmPlan& P = *w.P;
   const int u = w.h->cur[F];
   const int* src;
@@ -671,7 +729,7 @@ __device__ void frame_count(W& w, int m) {
 
 // fused mode at frame F = k-2: count over all remaining (sibling, candidate)
 // pairs, 32 jobs per pass.  Returns when the frame is exhausted.
-__device__ void fused_count(W& w, int F) {
+__device__ STEP_INL void fused_count(W& w, int F) {
   const StmPlan& P = *w.P;
   const bool lk = locked_frame(w, F);
   for (;;) {
@@ -756,6 +814,9 @@ __device__ __noinline__ bool try_chunk(W& w) {
   b = bcast(b);
   e = bcast(e);
   w.exhausted = __shfl_sync(FULLMASK, w.exhausted, 0);
+#if STM_PROFILE
+  if (b < 0 && w.first_dry == 0) w.first_dry = clock64();
+#endif
   if (b < 0) return false;
   lock_ws(w, w.h);
   if (w.lane == 0) {
@@ -1095,7 +1156,7 @@ __device__ volatile int* warp_sib(const W& w, int wid) {
 // ----------------------------------------------------------------------------
 // the kernel
 // ----------------------------------------------------------------------------
-__global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constant__ StmKParams kp) {
+__global__ void __launch_bounds__(STM_MAXT, 1) stm_count_kernel(const __grid_constant__ StmKParams kp) {
   extern __shared__ __align__(16) unsigned char smem[];
   const StmPlan& P = kp.plan;
   BlockHdr* bh = (BlockHdr*)smem;
@@ -1132,6 +1193,10 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
   w.steal_fails = 0;
   w.wbytes = w.wmerge = w.wjobs = 0;
   w.idle_cyc = 0;
+#if STM_PROFILE
+  for (int i = 0; i < STM_PROF_N; ++i) w.prof_cyc[i] = w.prof_cnt[i] = w.prof_items[i] = 0;
+  w.first_dry = 0;
+#endif
   if (lane == 0) {
     w.h->lock = 0;
     w.h->L = 0;
@@ -1158,14 +1223,18 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
     if (L == 0) {
       const bool lk = stealing(w);
       if (lk) lock_ws(w, w.h);
+      PROF_BEGIN(0)
       int m = gather_roots(w);
+      PROF_END(0, m)
       if (m > 0) {
         if (w.lane == 0) {
           w.h->nsib[1] = m;
           w.h->cur[1] = 0;
         }
         __syncwarp();
+        PROF_BEGIN(1)
         set_sibling(w, 1, 0);
+        PROF_END(1, 1)
         if (k == 2) {
           if (lk) unlock_ws(w, w.h);
           frame_count(w, m);  // counts N(root) per root
@@ -1179,7 +1248,9 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
         // instrumented launches: time spent acquiring work (cursor, stealing, idle
         // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
         const long long ta = kp.count_bytes ? clock64() : 0;
+        PROF_BEGIN(7)
         const bool got = acquire_work(w, t0);
+        PROF_END(7, got)
         if (kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
         if (!got) break;
       }
@@ -1187,7 +1258,9 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
     }
     const int F = L;
     if (fused && F == k - 2) {
+      PROF_BEGIN(5)
       fused_count(w, F);
+      PROF_END(5, 0)
       const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
       if (lk) lock_ws(w, w.h);
       if (w.lane == 0) w.h->L = F - 1;
@@ -1196,14 +1269,20 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
       continue;
     }
     const bool lk = locked_frame(w, F);
-    if (kp.global_steal && F < kp.detect_level && F < kp.stop_level) maybe_donate(w);
+    if (kp.global_steal && F < kp.detect_level && F < kp.stop_level) {
+      PROF_BEGIN(6)
+      maybe_donate(w);
+      PROF_END(6, 0)
+    }
     if (lk) lock_ws(w, w.h);
     int m = 0;
     bool back = false;
     for (;;) {
       if (w.h->cur[F] >= w.h->nsib[F]) { back = true; break; }
       if (w.h->it[F] < w.h->end[F]) {
+        PROF_BEGIN(2)
         m = gather_batch(w, F, U);
+        PROF_END(2, m)
         if (m > 0) break;
       }
       int nu = w.h->cur[F] + 1;
@@ -1213,7 +1292,9 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
         back = true;
         break;
       }
+      PROF_BEGIN(8)
       set_sibling(w, F, nu);
+      PROF_END(8, 1)
     }
     if (back) {
       if (w.lane == 0) w.h->L = F - 1;
@@ -1223,21 +1304,42 @@ __global__ void __launch_bounds__(1024, 1) stm_count_kernel(const __grid_constan
     }
     if (lk) unlock_ws(w, w.h);
     // build frame F+1 from the batch
+    PROF_BEGIN(3)
     build_nodes(w, F, m);
+    PROF_END(3, m)
     if (F + 1 == k - 1) {  // frame-count mode
+      PROF_BEGIN(4)
       frame_count(w, m);
+      PROF_END(4, m)
       continue;
     }
     const bool lk2 = locked_frame(w, F + 1);
     if (lk2) lock_ws(w, w.h);
     if (w.lane == 0) w.h->nsib[F + 1] = m;
     __syncwarp();
+    PROF_BEGIN(9)
     set_sibling(w, F + 1, 0);
+    PROF_END(9, 1)
     if (w.lane == 0) w.h->L = F + 1;
     __syncwarp();
     if (lk2) unlock_ws(w, w.h);
   }
   if (lane == 0 && w.cnt) atomicAdd(&kp.work->count, w.cnt);
+#if STM_PROFILE
+  if (lane == 0) {
+    for (int i = 0; i < STM_PROF_N; ++i) {
+      atomicAdd(&kp.work->prof[3 * i], w.prof_cyc[i]);
+      atomicAdd(&kp.work->prof[3 * i + 1], w.prof_cnt[i]);
+      atomicAdd(&kp.work->prof[3 * i + 2], w.prof_items[i]);
+    }
+    const long long now = clock64();
+    atomicAdd(&kp.work->prof[3 * STM_PROF_N], (unsigned long long)(now - t0));
+    // tail shape (clock64 is per SM; SMs start within a few us of each other)
+    atomicMax(&kp.work->prof[3 * STM_PROF_N + 1], (unsigned long long)(now - t0));
+    atomicAdd(&kp.work->prof[3 * STM_PROF_N + 2], (unsigned long long)(w.first_dry ? w.first_dry - t0 : now - t0));
+    atomicMax(&kp.work->prof[3 * STM_PROF_N + 3], (unsigned long long)(w.first_dry ? w.first_dry - t0 : now - t0));
+  }
+#endif
   if (kp.count_bytes) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {

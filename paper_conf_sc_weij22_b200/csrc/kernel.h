@@ -17,6 +17,12 @@ struct StmTask {
   int32_t prefix[STM_KMAX];
 };
 
+// phases of the STM_PROFILE build: 0 gather_roots, 1 root set_sibling, 2 gather_batch,
+// 3 build_nodes, 4 frame_count, 5 fused_count, 6 maybe_donate, 7 acquire_work,
+// 8 next-sibling set_sibling, 9 descend set_sibling, 10 run_jobs set-up (operand
+// narrowing), 11 run_jobs element loop (probes + compaction)
+#define STM_PROF_N 12
+
 // Device-resident scheduler state of one launch (zeroed before every launch).
 struct StmWork {
   unsigned long long count;       // result accumulator (mod 2^64)
@@ -28,6 +34,8 @@ struct StmWork {
   unsigned long long n_jobs;
   unsigned long long idle_cycles;  // sum over warps of cycles spent acquiring work (instrumented)
   unsigned long long warp_cycles;  // sum over warps of their lifetime in cycles (instrumented)
+  unsigned long long prof[3 * STM_PROF_N + 4];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
+                                                // lifetime, max lifetime, summed / max time cursors ran dry
 };
 
 struct StmBlockSlot {             // per block, global memory (Fig. 6)

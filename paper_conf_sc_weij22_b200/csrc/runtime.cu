@@ -21,6 +21,7 @@
 
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
+static thread_local uint64_t g_prof[3 * STM_PROF_N + 4] = {};
 
 stm_status stm_fail(stm_status s, const char* fmt, ...) {
   va_list ap;
@@ -365,7 +366,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->stop_level = 2;
   t->detect_level = 2;
   t->unroll = 8;
-  t->root_chunk = 32;
+  t->root_chunk = 2;  // measured on B200 (tools/gpu_tune.sh): 32 -> 2 is 1.5-1.8x on C2/C3, neutral on C5
   t->block_warps = 16;
   t->blocks_per_sm = 0;
 }
@@ -509,6 +510,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     g_info.merge_bytes = (int64_t)hw.merge_bytes;
     g_info.jobs = (int64_t)hw.n_jobs;
     g_info.idle_cycles = (int64_t)hw.idle_cycles;
+    memcpy(g_prof, hw.prof, sizeof g_prof);
     g_info.warp_cycles = (int64_t)hw.warp_cycles;
     *h_count = hw.count;
   }
@@ -548,6 +550,12 @@ extern "C" stm_status stm_match_count_per_root(const stm_graph* g, const stm_pla
   cudaFree(d);
   if (s == STM_OK) *count = c;
   return s;
+}
+
+extern "C" stm_status stm_last_profile(uint64_t* out, int n) {
+  if (!out || n < 0) return stm_fail(STM_EINVAL, "NULL out");
+  for (int i = 0; i < n && i < 3 * STM_PROF_N + 4; ++i) out[i] = g_prof[i];
+  return STM_OK;
 }
 
 extern "C" stm_status stm_last_launch(stm_launch_info* info) {

@@ -30,6 +30,22 @@ def shard_chunks(n: int, chunk: int, rank: int, world: int) -> List[int]:
     return list(range(rank, nchunks, world))
 
 
+def chunk_roots(c: int, chunk: int, n: int):
+    """Root-ID range [b, e) of chunk c (empty past the end)."""
+    b = min(n, c * chunk)
+    return b, min(n, b + chunk)
+
+
+def cursor_chunk(owner: int, idx: int, world: int) -> int:
+    """Chunk handed out by the idx-th atomicAdd on rank `owner`'s cursor (kernel try_chunk)."""
+    return owner + world * idx
+
+
+def steal_order(rank: int, world: int) -> List[int]:
+    """Cursors a rank's kernel draws from: its own first, then the peers' in ring order."""
+    return [(rank + i) % world for i in range(world)]
+
+
 class MultiGPUCounter:
     """Counts on this rank's GPU; combines ranks with one NCCL all-reduce."""
 

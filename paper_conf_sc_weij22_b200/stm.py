@@ -21,7 +21,7 @@ _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED
 EXPORTS = ["stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
            "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
            "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
-           "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_error"]
+           "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error"]
 
 
 class StmError(RuntimeError):
@@ -204,6 +204,21 @@ def stm_match_count_per_root(g: int, p: int, tuning: Optional[stm_tuning] = None
     c = ctypes.c_uint64()
     _check(lib.stm_match_count_per_root(g, p, _tp(tuning), stream, out.ctypes.data, ctypes.byref(c)))
     return c.value, out[:n]
+
+
+PROF_PHASES = ["gather_roots", "root_sibling", "gather_batch", "build_nodes", "frame_count", "fused_count",
+               "donate", "acquire_work", "next_sibling", "descend", "jobs_setup", "jobs_loop"]
+
+
+def stm_last_profile() -> dict:
+    N = 3 * len(PROF_PHASES) + 4
+    out = (ctypes.c_uint64 * N)()
+    _check(lib.stm_last_profile(out, N))
+    d = {ph: {"cycles": out[3 * i], "calls": out[3 * i + 1], "items": out[3 * i + 2]}
+         for i, ph in enumerate(PROF_PHASES)}
+    d["lifetime_cycles"] = out[N - 4]
+    d["tail"] = {"max_lifetime": out[N - 3], "sum_dry": out[N - 2], "max_dry": out[N - 1]}
+    return d
 
 
 def stm_last_launch() -> dict:

@@ -120,6 +120,7 @@ TUNINGS = [
     dict(root_chunk=1, stop_level=3, detect_level=3),
     dict(block_warps=4), dict(block_warps=32, blocks_per_sm=1),
     dict(vertex_order=1), dict(vertex_order=1, unroll=1, local_steal=0, global_steal=0),
+    dict(root_chunk=32), dict(root_chunk=7, unroll=3),
 ]
 
 
