@@ -293,20 +293,26 @@ def main():
     matches_per_step = sum(counts)
     value = matches_per_step * args.steps / (total_ms / 1000.0)
 
-    # ---- roofline of the (only) kernel: algorithmic bytes / average launch time
+    # ---- roofline of the dominant kernel (the query launch with the largest mean time):
+    # its algorithmic bytes W (one instrumented launch) / its mean
+    # CUDA-event launch time over the timed steps
     import json as _json
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
     if os.path.exists(peaks_path):
-        peak, peak_src = float(_json.load(open(peaks_path))["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+        pk = _json.load(open(peaks_path))
+        peak = float(pk.get("hbm_gbs_sustained", pk["hbm_gbs"]))
+        peak_src = "measured (MEASURED_PEAKS.json " + ("hbm_gbs_sustained" if "hbm_gbs_sustained" in pk else "hbm_gbs") + ")"
     avg_launch_s = [statistics.mean(x) / 1000.0 for x in launch_ms]
+    dom = max(range(len(plans)), key=lambda i: avg_launch_s[i])
     W_step = float(sum(alg))
-    achieved = W_step / sum(avg_launch_s) / 1e9
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", f"ncu_{args.workload}.json")
+    achieved = alg[dom] / avg_launch_s[dom] / 1e9
+    traffic, traffic_src = None, None
+    prof = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}_{queries[dom][0]}.json")
     if os.path.exists(prof):
         try:
-            traffic = _json.load(open(prof)).get("dram_bytes_per_launch")
+            pj = _json.load(open(prof))
+            traffic, traffic_src = pj.get("dram_bytes_per_launch"), os.path.relpath(prof, ROOT)
         except Exception:
             traffic = None
 
@@ -344,9 +350,13 @@ def main():
             "per_query": per_q,
             "gpu_launches": args.steps * len(plans),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "algorithmic_bytes_per_step": W_step,
-                         "note": "achieved = SURVEY.md 8(d) W (instrumented launch) / mean CUDA-event launch time"},
+                         "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                         "kernel": f"stm_count_kernel ({queries[dom][0]} launch)",
+                         "algorithmic_bytes_per_launch": alg[dom], "algorithmic_bytes_per_step": W_step,
+                         "peak_source": peak_src,
+                         "note": "achieved = SURVEY.md 8(d) W of the dominant launch (instrumented launch) / "
+                                 "its mean CUDA-event launch time; traffic = ncu dram read+write bytes of "
+                                 "that launch (--set full capture, committed under profiles/)"},
             "clocks": clk.summary(),
             "e2e": e2e,
             "cpu_baseline": cpu,

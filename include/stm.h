@@ -152,6 +152,12 @@ typedef struct stm_tuning {
                              breaks the symmetry), far less work on skewed graphs; per-root output
                              then attributes each match to f(order[0]) minimal in (degree, id) order.
                              1 = always the caller's vertex ids.  Default 0. */
+  int32_t bitmap_min_degree; /* hub adjacency bitmaps (B200 design choice):
+                             every vertex of degree >= this gets an n-bit bitmap of its neighbour list
+                             in HBM, and set-operation probes into its list test one bit instead of
+                             binary-searching.  0 = auto (64), -1 = off.  Built lazily on the first
+                             launch that uses them and cached on the graph.  Speed only. */
+  int32_t bitmap_budget_mb;  /* at most this many MiB of bitmaps (highest degrees first); 0 = auto (2048). */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -230,6 +236,7 @@ typedef struct stm_launch_info {
                               waiting idle); instrumented calls only */
   int64_t warp_cycles;     /* sum over warps of their lifetime in SM cycles; instrumented calls only.
                               idle_cycles / warp_cycles = idle/stealing fraction of warps */
+  int64_t hubs;            /* vertices with a hub adjacency bitmap in the counted numbering */
 } stm_launch_info;
 
 stm_status stm_last_launch(stm_launch_info* info);

@@ -165,6 +165,10 @@ __device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) 
   p = w.kp->col_idx + b;
   len = (int)(e - b);
 }
+// bitmap slot of v's neighbour list, -1 when v has none
+__device__ __forceinline__ int hslot(const W& w, int v) {
+  return w.kp->hub_slot ? w.kp->hub_slot[v] : -1;
+}
 __device__ __forceinline__ int degree(const W& w, int v) {
   return (int)(w.kp->row_ptr[v + 1] - w.kp->row_ptr[v]);
 }
@@ -253,6 +257,7 @@ struct Job {
   int* out;      // materialise target (NULL in count mode)
   int u, c;      // context for exclusions / per-root attribution
   int a_node;    // 0: A is a CSR row; l+1: A is an arena set node of level l (rebuilt with its frame)
+  int abm, bbm;  // hub bitmap slot of A (if a CSR row) / of B, -1 = none
 };
 
 __device__ __forceinline__ void narrow(const int*& p, int& n, int lo, int hi) {
@@ -325,13 +330,19 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   const int* D = An;
   const int* Pp = Bn;
   int dlen = an, plen = bn, use_h = 0;
+  int pslot = -1;  // bitmap slot of the probed operand
   if (mine) {
-    if (J.op == STM_OP_AND && bn < an) { D = Bn; dlen = bn; Pp = An; plen = an; }
-    if (!J.B) { Pp = nullptr; plen = 0; }
+    pslot = J.bbm;
+    if (J.op == STM_OP_AND && bn < an) { D = Bn; dlen = bn; Pp = An; plen = an; pslot = J.abm; }
+    if (!J.B) { Pp = nullptr; plen = 0; pslot = -1; }
+    // a probed hub row is tested in its bitmap: one word per element instead of
+    // ceil(log2 |P|) dependent loads (the driving element already lies in (lo, hi))
+    if (pslot >= 0) Pp = (const int*)(w.kp->bitmaps + (size_t)pslot * (size_t)w.kp->bm_words);
     if (hmode) {
       const int dh = hmode == 1 ? bn : an;
       if (dh * 2 <= dlen * (log2c(plen) + 1) * 4) {
         use_h = 1;
+        pslot = -1;
         if (hmode == 1) { D = Bn; dlen = bn; } else { D = An; dlen = an; }
       }
     }
@@ -355,7 +366,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   }
   const int total = __shfl_sync(FULLMASK, incl, 31);
   const int start = incl - dlen;
-  const int flags = (Pp != nullptr ? 1 : 0) | (use_h ? 2 : 0) | (J.op == STM_OP_DIFF ? 4 : 0);
+  const int flags = (Pp != nullptr ? 1 : 0) | (use_h ? 2 : 0) | (J.op == STM_OP_DIFF ? 4 : 0) | (pslot >= 0 ? 8 : 0);
   const int* const ht = w.ht;
   const unsigned htmask = w.ht_mask;
   const uint8_t* const glabels = w.kp->labels;
@@ -387,7 +398,10 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       x = Dj[e - sj];
       keep = x > loj && x < hij;
       if (keep && (fj & 1)) {
-        const bool f = (STM_WITH_HASH && (fj & 2)) ? ht_has(ht, htmask, x) : member(Pj, pl, x);
+        bool f;
+        if (fj & 8) f = (__ldg((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
+        else if (STM_WITH_HASH && (fj & 2)) f = ht_has(ht, htmask, x);
+        else f = member(Pj, pl, x);
         keep = (fj & 4) ? !f : f;
       }
       if (keep && labj != STM_LAB_ANY) keep = (l2s[glabels[x]] & labj) != 0;
@@ -451,7 +465,13 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   J.B = nullptr;
   J.blen = 0;
   J.op = P.cnt_op;
-  if (P.cnt_op != STM_OP_NONE) row(w, pval(w, P.cnt_b, F, u, c), J.B, J.blen);
+  J.abm = P.cnt_a.kind == STM_SRC_RAW ? hslot(w, pval(w, P.cnt_a.idx, F, u, c)) : -1;
+  J.bbm = -1;
+  if (P.cnt_op != STM_OP_NONE) {
+    const int vb = pval(w, P.cnt_b, F, u, c);
+    row(w, vb, J.B, J.blen);
+    J.bbm = hslot(w, vb);
+  }
   const StmFilter f = P.filt[P.k - 1];
   bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
   J.lab = f.lab;
@@ -548,6 +568,23 @@ __device__ int node_ub(const W& w, int s, int F, int u, int c) {
   }
 }
 
+// The part of node_ub that does not depend on the candidate (position F) of frame
+// F, sibling u: INT_MAX when every term does.
+__device__ int node_ub_const(const W& w, int s, int F, int u) {
+  const StmPlan& P = *w.P;
+  int m = INT_MAX;
+  for (;;) {
+    const StmNode nd = P.nodes[s];
+    if (nd.op == STM_OP_AND && nd.b != F) m = min(m, degree(w, pval(w, nd.b, F, u, 0)));
+    if (nd.a_kind == STM_SRC_RAW) return nd.a != F ? min(m, degree(w, pval(w, nd.a, F, u, 0))) : m;
+    if (P.nodes[nd.a].level == F + 1) { s = nd.a; continue; }
+    const int* p;
+    int len;
+    node_slice(w, nd.a, F, u, 0, p, len);
+    return min(m, len);
+  }
+}
+
 // Compute the nodes of level F+1 for the m siblings SIB(F+1, 0..m-1); offsets
 // NOFF were assigned by the caller; sizes NSZ are written here.
 __device__ STEP_INL void build_nodes(W& w, int F, int m) {
@@ -569,7 +606,7 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
       const int nj = min(32, njobs_total - j0);
       Job J;
       J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_AND;
-      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0;
+      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
       int s = 0, t = 0;
       if (w.lane < nj) {
         s = nodes_in[jj / m];
@@ -577,10 +614,17 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
         const StmNode nd = P.nodes[s];
         const int c = SIB(w, F + 1, t);
         J.c = c;
-        if (nd.a_kind == STM_SRC_RAW) row(w, pval(w, nd.a, F, u, c), J.A, J.alen);
-        else node_slice(w, nd.a, F, u, t, J.A, J.alen);
+        if (nd.a_kind == STM_SRC_RAW) {
+          const int va = pval(w, nd.a, F, u, c);
+          row(w, va, J.A, J.alen);
+          J.abm = hslot(w, va);
+        } else {
+          node_slice(w, nd.a, F, u, t, J.A, J.alen);
+        }
         J.a_node = nd.a_kind == STM_SRC_NODE ? P.nodes[nd.a].level + 1 : 0;
-        row(w, pval(w, nd.b, F, u, c), J.B, J.blen);
+        const int vb = pval(w, nd.b, F, u, c);
+        row(w, vb, J.B, J.blen);
+        J.bbm = hslot(w, vb);
         J.op = nd.op;
         bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
         J.lab = nd.lab;
@@ -612,6 +656,39 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
   const int e = w.h->end[F];
   const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
   const int cap = w.kp->cap;
+  // Fast admission: when U copies of every node's candidate-independent size bound
+  // fit in its region, any batch of <= U candidates fits -- fixed slice offsets
+  // t * bound, no per-candidate degree loads or prefix sums.
+  bool fixed = true;
+  for (int s = nb; s < ne && fixed; ++s) fixed = (long long)node_ub_const(w, s, F, u) * U <= (long long)cap;
+  if (fixed) {
+    int m = 0;
+    while (m < U && pos < e) {
+      const int p = pos + w.lane;
+      const bool valid = p < e;
+      const int c = valid ? src[p] : 0;
+      const bool pass = valid && cand_ok(w, F, u, c, lo, hi);
+      unsigned acc = __ballot_sync(FULLMASK, pass);
+      const int room = U - m;
+      bool cut = false;
+      if (__popc(acc) > room) {
+        unsigned a2 = 0, t = acc;  // keep the first `room` set bits
+        for (int i = 0; i < room; ++i) { const unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+        acc = a2;
+        cut = true;
+      }
+      if ((acc >> w.lane) & 1u) SIB(w, F + 1, m + __popc(acc & ((1u << w.lane) - 1))) = c;
+      m += __popc(acc);
+      pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+    }
+    for (int s = nb; s < ne; ++s) {
+      const int ub0 = node_ub_const(w, s, F, u);
+      if (w.lane < m) NOFF(w, s, w.lane) = w.lane * ub0;
+    }
+    if (w.lane == 0) w.h->it[F] = pos;
+    __syncwarp();
+    return m;
+  }
   if (w.lane == 0)
     for (int s = nb; s < ne; ++s) w.h->used[s] = 0;
   __syncwarp();
@@ -722,7 +799,7 @@ __device__ void frame_count(W& w, int m) {
   const int u = F >= 1 ? w.h->cur[F] : 0;
   Job J;
   J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
-  J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0;
+  J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
   if (w.lane < m) J = count_job(w, F, u, SIB(w, k - 1, w.lane), w.lane);
   w.cnt += run_jobs(w, J, m, true, F, w.P->filt[k - 1].excl, nullptr);
 }
@@ -783,7 +860,7 @@ __device__ STEP_INL void fused_count(W& w, int F) {
     if (nj == 0) return;
     Job J;
     J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
-    J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0; J.a_node = 0;
+    J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
     if (w.lane < nj) J = count_job(w, F, w.h->stage_u[w.lane], w.h->stage_c[w.lane], 0);
     w.cnt += run_jobs(w, J, nj, true, F, P.filt[P.k - 1].excl, nullptr);
     __syncwarp();

@@ -50,6 +50,12 @@ struct StmKParams {
   const int64_t* row_ptr;
   const int32_t* col_idx;
   const uint8_t* labels;          // dense graph label ids, or NULL
+  // Hub adjacency bitmaps: hub_slot[v] >= 0 selects the
+  // n-bit row bitmaps[slot * bm_words ...] of N(v); membership probes into such a
+  // row read one word instead of a binary search.  hub_slot == NULL: none.
+  const int32_t* hub_slot;
+  const uint32_t* bitmaps;
+  int64_t bm_words;
   int64_t n;
   int32_t cap;                    // words per set-node region per warp
   int32_t block_warps;

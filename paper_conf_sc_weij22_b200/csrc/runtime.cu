@@ -19,6 +19,10 @@
 #include "internal.h"
 #include "kernel.h"
 
+// Hub bitmap defaults (stm_tuning 0 = auto): measured on B200, DESIGN.md "Hub bitmaps".
+#define STM_BITMAP_AUTO_MIN_DEGREE 64
+#define STM_BITMAP_AUTO_BUDGET_MB 2048
+
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
 static thread_local uint64_t g_prof[3 * STM_PROF_N + 4] = {};
@@ -79,6 +83,15 @@ struct stm_graph {
   int32_t* d_rcol_idx = nullptr;
   uint8_t* d_rlabels = nullptr;
   int32_t* d_rank2orig = nullptr;  // [n]: ranked id -> caller's id (per-root output)
+  // Hub adjacency bitmaps, per numbering ([0] caller's ids, [1] degree-ranked),
+  // built lazily by the first launch that asks for them.
+  struct HubBitmaps {
+    int32_t* slot = nullptr;   // [n]: bitmap slot of v, -1 = none
+    uint32_t* bits = nullptr;  // [n_hubs][words]
+    int64_t words = 0, n_hubs = 0;
+    int min_deg = -2;          // parameters the cached copy was built with (-2 = never built)
+    int64_t budget = -1;
+  } hub[2];
   std::mutex mu;
   std::map<void*, Scratch> scratch;  // per stream
 };
@@ -181,6 +194,90 @@ static void build_ranked(stm_graph* g) {
   g->d_rrow_ptr = nullptr;
   g->d_rcol_idx = nullptr;
   g->d_rlabels = nullptr;
+}
+
+// ---------------------------------------------------------------- hub bitmaps
+__global__ void count_deg_ge(const int64_t* rp, int64_t n, int64_t min_deg, unsigned long long* out) {
+  unsigned long long c = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    c += (rp[v + 1] - rp[v]) >= min_deg;
+  if (c) atomicAdd(out, c);
+}
+// hub i is the vertex of ranked id n - H + i (the H highest in (degree, id) order)
+__global__ void hub_slots(int64_t n, int64_t H, const int32_t* rank2orig, int32_t* slot) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < H; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = n - H + i;
+    slot[rank2orig ? rank2orig[r] : r] = (int32_t)i;
+  }
+}
+// one block per hub: set the bits of its neighbour list
+__global__ void hub_fill(int64_t n, int64_t H, const int32_t* rank2orig, const int64_t* rp, const int32_t* ci,
+                         int64_t words, uint32_t* bits) {
+  for (int64_t i = blockIdx.x; i < H; i += gridDim.x) {
+    const int64_t r = n - H + i;
+    const int32_t v = rank2orig ? rank2orig[r] : (int32_t)r;
+    uint32_t* b = bits + (size_t)i * (size_t)words;
+    for (int64_t e = rp[v] + threadIdx.x; e < rp[v + 1]; e += blockDim.x) {
+      const int32_t x = ci[e];
+      atomicOr(&b[x >> 5], 1u << (x & 31));
+    }
+  }
+}
+
+static void free_hub(stm_graph::HubBitmaps& h) {
+  cudaFree(h.slot);
+  cudaFree(h.bits);
+  h = stm_graph::HubBitmaps();
+}
+
+// Makes g->hub[ranked] hold bitmaps of every vertex with degree >= min_deg, at most
+// budget bytes (highest degrees first).  Speed only: on any failure there are none.
+static const stm_graph::HubBitmaps* ensure_hub(stm_graph* g, bool ranked, int min_deg, int64_t budget) {
+  stm_graph::HubBitmaps& h = g->hub[ranked ? 1 : 0];
+  if (min_deg < 0 || !g->ranked || g->n < 1) return nullptr;
+  if (h.min_deg == min_deg && h.budget == budget) return h.n_hubs ? &h : nullptr;
+  free_hub(h);
+  h.min_deg = min_deg;
+  h.budget = budget;
+  const int64_t n = g->n;
+  const int64_t words = (n + 31) / 32;
+  const int64_t hmax = budget / (words * 4);
+  unsigned long long* d = nullptr;
+  unsigned long long H = 0;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 4096);
+  cudaError_t e = cudaMalloc(&d, sizeof H);
+  if (e == cudaSuccess) e = cudaMemset(d, 0, sizeof H);
+  if (e == cudaSuccess) count_deg_ge<<<grid, 256>>>(g->d_rrow_ptr, n, std::max(min_deg, 1), d);
+  if (e == cudaSuccess) e = cudaMemcpy(&H, d, sizeof H, cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  H = std::min<unsigned long long>(H, (unsigned long long)std::max<int64_t>(hmax, 0));
+  if (e != cudaSuccess || H == 0) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  e = cudaMalloc(&h.slot, sizeof(int32_t) * n);
+  if (e == cudaSuccess) e = cudaMalloc(&h.bits, sizeof(uint32_t) * (size_t)words * H);
+  if (e == cudaSuccess) e = cudaMemset(h.slot, 0xFF, sizeof(int32_t) * n);
+  if (e == cudaSuccess) e = cudaMemset(h.bits, 0, sizeof(uint32_t) * (size_t)words * H);
+  if (e == cudaSuccess) {
+    const int32_t* r2o = ranked ? nullptr : g->d_rank2orig;
+    hub_slots<<<(unsigned)std::min<unsigned long long>((H + 255) / 256, 4096), 256>>>(n, (int64_t)H, r2o, h.slot);
+    hub_fill<<<(unsigned)std::min<unsigned long long>(H, 65535), 256>>>(
+        n, (int64_t)H, r2o, ranked ? g->d_rrow_ptr : g->d_row_ptr, ranked ? g->d_rcol_idx : g->d_col_idx, words,
+        h.bits);
+    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    free_hub(h);
+    h.min_deg = min_deg;
+    h.budget = budget;
+    return nullptr;
+  }
+  h.words = words;
+  h.n_hubs = (int64_t)H;
+  return &h;
 }
 
 static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci) {
@@ -354,6 +451,8 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
   cudaFree(g->d_rrow_ptr);
   cudaFree(g->d_rcol_idx);
   cudaFree(g->d_rlabels);
+  free_hub(g->hub[0]);
+  free_hub(g->hub[1]);
   delete g;
   return STM_OK;
 }
@@ -369,6 +468,8 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->root_chunk = 2;  // measured on B200 (tools/gpu_tune.sh): 32 -> 2 is 1.5-1.8x on C2/C3, neutral on C5
   t->block_warps = 16;
   t->blocks_per_sm = 0;
+  t->bitmap_min_degree = 0;  // auto
+  t->bitmap_budget_mb = 0;   // auto
 }
 
 // ---------------------------------------------------------------------------- match
@@ -407,6 +508,16 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.labels = use_rank ? g->d_rlabels : g->d_labels;
   kp.root_map = use_rank ? g->d_rank2orig : nullptr;
   kp.n = g->n;
+  {
+    const int min_deg = t.bitmap_min_degree == 0 ? STM_BITMAP_AUTO_MIN_DEGREE : t.bitmap_min_degree;
+    const int64_t budget = (int64_t)(t.bitmap_budget_mb > 0 ? t.bitmap_budget_mb : STM_BITMAP_AUTO_BUDGET_MB) << 20;
+    std::lock_guard<std::mutex> lk(g->mu);
+    const stm_graph::HubBitmaps* hb = ensure_hub(g, use_rank, min_deg, budget);
+    kp.hub_slot = hb ? hb->slot : nullptr;
+    kp.bitmaps = hb ? hb->bits : nullptr;
+    kp.bm_words = hb ? hb->words : 0;
+    g_info.hubs = hb ? hb->n_hubs : 0;
+  }
   // label-slot table: dense graph label -> bitmask of pattern slots with that value
   for (int d = 0; d < (int)g->label_values.size(); ++d)
     for (int s = 0; s < P.n_label_slots; ++s)

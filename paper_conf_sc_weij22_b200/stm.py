@@ -33,7 +33,8 @@ class StmError(RuntimeError):
 class stm_tuning(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("local_steal", "global_steal", "stop_level", "detect_level",
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
-                                               "instrument", "hash_slots", "vertex_order")]
+                                               "instrument", "hash_slots", "vertex_order",
+                                               "bitmap_min_degree", "bitmap_budget_mb")]
 
 
 class stm_shard(ctypes.Structure):
@@ -46,7 +47,8 @@ class stm_launch_info(ctypes.Structure):
                 ("cap", ctypes.c_int32), ("arena_bytes", ctypes.c_int64), ("local_steals", ctypes.c_int64),
                 ("global_steals", ctypes.c_int64), ("chunks", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("merge_bytes", ctypes.c_int64), ("jobs", ctypes.c_int64), ("ranked", ctypes.c_int32),
-                ("reserved", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64)]
+                ("reserved", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64),
+                ("hubs", ctypes.c_int64)]
 
 
 def _load():

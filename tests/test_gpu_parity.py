@@ -121,7 +121,26 @@ TUNINGS = [
     dict(block_warps=4), dict(block_warps=32, blocks_per_sm=1),
     dict(vertex_order=1), dict(vertex_order=1, unroll=1, local_steal=0, global_steal=0),
     dict(root_chunk=32), dict(root_chunk=7, unroll=3),
+    dict(bitmap_min_degree=1), dict(bitmap_min_degree=-1), dict(bitmap_min_degree=1, vertex_order=1),
+    dict(bitmap_min_degree=40, unroll=1),
 ]
+
+
+@pytest.mark.parametrize("name", SMALL + ["k6_minus_e", "octahedron", "w5"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_hub_bitmaps(rmat_small, name, vi):
+    """Hub bitmaps (every vertex, caller's and degree-ranked numbering, labeled and not)
+    change only how membership is probed, never the count."""
+    g, G = rmat_small
+    p = CATALOG[name]
+    want = ocount(g, p, vi)
+    for vo in (0, 1):
+        t = stm.stm_tuning_default(bitmap_min_degree=1, vertex_order=vo)
+        assert gcount(G, p, vi, tuning=t) == want, (name, vi, vo)
+        assert stm.stm_last_launch()["hubs"] > 0
+    pl = tuple(int(x) for x in np.random.default_rng(p.k).integers(0, 4, p.k))
+    t = stm.stm_tuning_default(bitmap_min_degree=8)
+    assert gcount(G, p, vi, pl, tuning=t) == ocount(g, p, vi, pl)
 
 
 @pytest.mark.parametrize("tk", range(len(TUNINGS)))
