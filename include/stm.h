@@ -139,7 +139,8 @@ typedef struct stm_tuning {
   int32_t global_steal;   /* 0/1: inter-block stealing through global mailboxes (Sec. V-B). Default 1. */
   int32_t stop_level;     /* frames < stop_level are stealable (paper: 2). Default 2. */
   int32_t detect_level;   /* donors look for idle blocks at frames < detect_level (paper: 1). Default 2. */
-  int32_t unroll;         /* sibling iterations expanded together, 1..16 (paper: 8). Default 8. */
+  int32_t unroll;         /* sibling iterations expanded together, 1..32 (paper: 8);
+                             0 = auto (32 with the 40-register kernel, else 16; measured).  Default 0. */
   int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 2 (measured best on B200). */
   int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
@@ -158,6 +159,12 @@ typedef struct stm_tuning {
                              binary-searching.  0 = auto (64), -1 = off.  Built lazily on the first
                              launch that uses them and cached on the graph.  Speed only. */
   int32_t bitmap_budget_mb;  /* at most this many MiB of bitmaps (highest degrees first); 0 = auto (2048). */
+  int32_t occupancy;      /* kernel register budget: 1 = 64 registers (32 warps/SM), 2 = 40 registers
+                             (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
+                             than half the L2.  Speed only.  Default 0. */
+  int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
+                             out_start[v] (first neighbour > v, built at load); 1 = binary search only.
+                             Speed only.  Default 0. */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -237,6 +244,8 @@ typedef struct stm_launch_info {
   int64_t warp_cycles;     /* sum over warps of their lifetime in SM cycles; instrumented calls only.
                               idle_cycles / warp_cycles = idle/stealing fraction of warps */
   int64_t hubs;            /* vertices with a hub adjacency bitmap in the counted numbering */
+  int32_t variant;         /* kernel variant launched (stm_tuning.occupancy: 1 or 2) */
+  int32_t unroll;          /* unroll factor used */
 } stm_launch_info;
 
 stm_status stm_last_launch(stm_launch_info* info);

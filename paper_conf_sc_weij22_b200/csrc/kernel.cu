@@ -56,6 +56,17 @@
 #else
 #define STEP_INL
 #endif
+#ifndef STM_ILP2
+#define STM_ILP2 0          // 1: element loop handles two 32-element slices per iteration (probe ILP)
+#endif
+#ifndef STM_INSTR
+#define STM_INSTR 0         // 1: the instrumented build (kernel_instr.cu): algorithmic-byte / idle counters
+#endif
+#if STM_INSTR
+#define STM_SYM(x) x##_instr
+#else
+#define STM_SYM(x) x
+#endif
 #ifndef STM_PROFILE
 #define STM_PROFILE 0       // 1: per-phase clock64() buckets (stm_last_profile); A/B builds only
 #endif
@@ -158,6 +169,21 @@ __device__ __forceinline__ bool member(const int* __restrict__ a, int n, int x) 
     n -= half;
   }
   return *base == x;
+}
+
+// Two independent membership searches interleaved (element-loop ILP): the dependent
+// probe chains of two elements overlap instead of running back to back.
+__device__ __forceinline__ void member2(const int* __restrict__ pa, int na, int xa, const int* __restrict__ pb,
+                                        int nb, int xb, bool& fa, bool& fb) {
+  const int* ba = pa;
+  const int* bb = pb;
+  int ra = na, rb = nb;
+  while (ra > 1 || rb > 1) {
+    if (ra > 1) { const int h = ra >> 1; ba = (ba[h] <= xa) ? ba + h : ba; ra -= h; }
+    if (rb > 1) { const int h = rb >> 1; bb = (bb[h] <= xb) ? bb + h : bb; rb -= h; }
+  }
+  fa = na > 0 && *ba == xa;
+  fb = nb > 0 && *bb == xb;
 }
 
 __device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) {
@@ -267,6 +293,26 @@ __device__ __forceinline__ void narrow(const int*& p, int& n, int lo, int hi) {
   }
 }
 
+// Narrow the CSR row p[0..n) of vertex v to the open interval (lo, hi) at job
+// construction.  out_start[v] splits the sorted row at v (p[0..s) < v < p[s..n)),
+// so the bound lo = v (the common case v_{l-1} < w of a restriction chain) costs one
+// load and every other bound searches only one side of the split.
+__device__ __forceinline__ void narrow_row(const W& w, int v, const int*& p, int& n, int lo, int hi) {
+  if (lo < 0 && hi == INT_MAX) return;
+  if (!w.kp->out_start) { narrow(p, n, lo, hi); return; }
+  const int s = w.kp->out_start[v];
+  const bool big = n > 16;
+  int b = 0, e = n;
+  if (lo >= v) { b = s; if (lo > v && big) b += lbound(p + s, n - s, lo + 1); }
+  else if (lo >= 0 && big) b = lbound(p, s, lo + 1);
+  if (hi <= v) { e = s; if (hi < v && big) e = lbound(p, s, hi); }
+  else if (hi < INT_MAX && big && hi > v + 1) e = s + lbound(p + s, n - s, hi);
+  else if (hi == v + 1) e = s;
+  e = max(e, b);
+  p += b;
+  n = e - b;
+}
+
 __device__ __forceinline__ int log2c(int n) { return 32 - __clz(n); }  // ceil(log2(n+1))
 
 // Returns the (warp-uniform) number of kept elements summed over all jobs when
@@ -281,10 +327,8 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   int an = mine ? J.alen : 0;
   const int* Bn = J.B;
   int bn = (mine && J.B) ? J.blen : 0;
-  if (mine) {
-    narrow(An, an, J.lo, J.hi);
-    if (J.B) narrow(Bn, bn, J.lo, J.hi);
-  }
+  // CSR-row operands were narrowed at job construction (narrow_row); arena sets here
+  if (mine && J.a_node) narrow(An, an, J.lo, J.hi);
   // ---- shared operand -> shared-memory hash set
   const unsigned long long a0 = __shfl_sync(FULLMASK, (unsigned long long)J.A, 0);
   const unsigned long long b0 = __shfl_sync(FULLMASK, (unsigned long long)J.B, 0);
@@ -347,7 +391,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       }
     }
   }
-  if (w.kp->count_bytes && mine) {
+  if (STM_INSTR && w.kp->count_bytes && mine) {
     // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below),
     // with A the driving operand and B the probed one (before hashing).
     int d, pl;
@@ -375,6 +419,75 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   unsigned long long jc = 0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
                            Oll = (unsigned long long)J.out;
+#if STM_ILP2
+  // two 32-element slices per iteration: slice h covers elements e0 + 32h + lane
+  for (int e0 = 0; e0 < total; e0 += 64) {
+    int j[2], x[2], fjs[2];
+    const int* Pjs[2];
+    int pls[2];
+    bool keep[2], need[2];
+    unsigned labjs[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int e = e0 + 32 * h + lane;
+      int jj = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        int v = __shfl_sync(FULLMASK, incl, jj + step - 1);
+        if (v <= e) jj += step;
+      }
+      j[h] = jj;
+      const bool valid = e < total;
+      const int* Dj = (const int*)__shfl_sync(FULLMASK, Dll, jj);
+      Pjs[h] = (const int*)__shfl_sync(FULLMASK, Pll, jj);
+      const int sj = __shfl_sync(FULLMASK, start, jj);
+      pls[h] = __shfl_sync(FULLMASK, plen, jj);
+      fjs[h] = __shfl_sync(FULLMASK, flags, jj);
+      const int loj = __shfl_sync(FULLMASK, J.lo, jj);
+      const int hij = __shfl_sync(FULLMASK, J.hi, jj);
+      labjs[h] = __shfl_sync(FULLMASK, J.lab, jj);
+      x[h] = valid ? Dj[e - sj] : 0;
+      keep[h] = valid && x[h] > loj && x[h] < hij;
+      need[h] = keep[h] && (fjs[h] & 1);
+    }
+    bool f[2] = {false, false};
+    bool bs[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      bs[h] = need[h] && !(fjs[h] & 8);
+      if (need[h] && (fjs[h] & 8)) f[h] = (__ldg((const unsigned*)Pjs[h] + (x[h] >> 5)) >> (x[h] & 31)) & 1u;
+    }
+    if (bs[0] || bs[1]) {
+      bool f0, f1;
+      member2(Pjs[0], bs[0] ? pls[0] : 0, x[0], Pjs[1], bs[1] ? pls[1] : 0, x[1], f0, f1);
+      if (bs[0]) f[0] = f0;
+      if (bs[1]) f[1] = f1;
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      if (need[h]) keep[h] = (fjs[h] & 4) ? !f[h] : f[h];
+      if (keep[h] && labjs[h] != STM_LAB_ANY) keep[h] = (l2s[glabels[x[h]]] & labjs[h]) != 0;
+      const int eb = e0 + 32 * h;
+      const unsigned km = __ballot_sync(FULLMASK, keep[h]);
+      int a = start - eb, b = incl - eb;
+      a = a < 0 ? 0 : a;
+      b = b > 32 ? 32 : b;
+      unsigned rmask = 0;
+      if (mine && a < b) rmask = (b == 32 ? FULLMASK : ((1u << b) - 1)) & ~((1u << a) - 1);
+      if (count_mode) {
+        jc += __popc(km & rmask);
+      } else {
+        int* Oj = (int*)__shfl_sync(FULLMASK, Oll, j[h]);
+        int base = __shfl_sync(FULLMASK, outc, j[h]);
+        int fl = __shfl_sync(FULLMASK, start, j[h]) - eb;
+        fl = fl < 0 ? 0 : fl;
+        unsigned before = km & ((1u << lane) - 1) & ~((1u << fl) - 1);
+        if (keep[h]) Oj[base + __popc(before)] = x[h];
+        outc += __popc(km & rmask);
+      }
+    }
+  }
+#else
   for (int e0 = 0; e0 < total; e0 += 32) {
     const int e = e0 + lane;
     int j = 0;
@@ -425,9 +538,10 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       outc += __popc(km & rmask);
     }
   }
+#endif
   PROF_END(11, total)
   if (!count_mode) {
-    if (w.kp->count_bytes && mine) w.wbytes += 4ull * (unsigned long long)outc;
+    if (STM_INSTR && w.kp->count_bytes && mine) w.wbytes += 4ull * (unsigned long long)outc;
     *outc_lane = outc;
     return 0;
   }
@@ -465,15 +579,21 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   J.B = nullptr;
   J.blen = 0;
   J.op = P.cnt_op;
-  J.abm = P.cnt_a.kind == STM_SRC_RAW ? hslot(w, pval(w, P.cnt_a.idx, F, u, c)) : -1;
+  const StmFilter f = P.filt[P.k - 1];
+  bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
+  J.abm = -1;
+  if (P.cnt_a.kind == STM_SRC_RAW) {
+    const int va = pval(w, P.cnt_a.idx, F, u, c);
+    J.abm = hslot(w, va);
+    narrow_row(w, va, J.A, J.alen, J.lo, J.hi);
+  }
   J.bbm = -1;
   if (P.cnt_op != STM_OP_NONE) {
     const int vb = pval(w, P.cnt_b, F, u, c);
     row(w, vb, J.B, J.blen);
     J.bbm = hslot(w, vb);
+    narrow_row(w, vb, J.B, J.blen, J.lo, J.hi);
   }
-  const StmFilter f = P.filt[P.k - 1];
-  bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
   J.lab = f.lab;
   J.out = nullptr;
   J.u = u;
@@ -614,10 +734,12 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
         const StmNode nd = P.nodes[s];
         const int c = SIB(w, F + 1, t);
         J.c = c;
+        bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
         if (nd.a_kind == STM_SRC_RAW) {
           const int va = pval(w, nd.a, F, u, c);
           row(w, va, J.A, J.alen);
           J.abm = hslot(w, va);
+          narrow_row(w, va, J.A, J.alen, J.lo, J.hi);
         } else {
           node_slice(w, nd.a, F, u, t, J.A, J.alen);
         }
@@ -625,8 +747,8 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
         const int vb = pval(w, nd.b, F, u, c);
         row(w, vb, J.B, J.blen);
         J.bbm = hslot(w, vb);
+        narrow_row(w, vb, J.B, J.blen, J.lo, J.hi);
         J.op = nd.op;
-        bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
         J.lab = nd.lab;
         J.out = w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
       }
@@ -1233,7 +1355,7 @@ __device__ volatile int* warp_sib(const W& w, int wid) {
 // ----------------------------------------------------------------------------
 // the kernel
 // ----------------------------------------------------------------------------
-__global__ void __launch_bounds__(STM_MAXT, 1) stm_count_kernel(const __grid_constant__ StmKParams kp) {
+__device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
   extern __shared__ __align__(16) unsigned char smem[];
   const StmPlan& P = kp.plan;
   BlockHdr* bh = (BlockHdr*)smem;
@@ -1324,11 +1446,11 @@ __global__ void __launch_bounds__(STM_MAXT, 1) stm_count_kernel(const __grid_con
       if (m == 0) {
         // instrumented launches: time spent acquiring work (cursor, stealing, idle
         // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
-        const long long ta = kp.count_bytes ? clock64() : 0;
+        const long long ta = (STM_INSTR && kp.count_bytes) ? clock64() : 0;
         PROF_BEGIN(7)
         const bool got = acquire_work(w, t0);
         PROF_END(7, got)
-        if (kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
+        if (STM_INSTR && kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
         if (!got) break;
       }
       continue;
@@ -1417,7 +1539,7 @@ __global__ void __launch_bounds__(STM_MAXT, 1) stm_count_kernel(const __grid_con
     atomicMax(&kp.work->prof[3 * STM_PROF_N + 3], (unsigned long long)(w.first_dry ? w.first_dry - t0 : now - t0));
   }
 #endif
-  if (kp.count_bytes) {
+  if (STM_INSTR && kp.count_bytes) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
       w.wbytes += __shfl_xor_sync(FULLMASK, w.wbytes, o);
@@ -1434,21 +1556,38 @@ __global__ void __launch_bounds__(STM_MAXT, 1) stm_count_kernel(const __grid_con
   }
 }
 
+// Two register budgets of the same kernel (stm_tuning.occupancy): 64 registers ->
+// 32 resident warps per SM, or 40 registers (with spills) -> 48 warps per SM, which
+// hides more DRAM latency when the graph does not fit in L2 (measured).
+__global__ void __launch_bounds__(STM_MAXT, 1) STM_SYM(stm_count_kernel)(const __grid_constant__ StmKParams kp) {
+  stm_count_body(kp);
+}
+__global__ void __launch_bounds__(1536, 1) STM_SYM(stm_count_kernel_occ)(const __grid_constant__ StmKParams kp) {
+  stm_count_body(kp);
+}
+
+static const void* STM_SYM(kernel_fn)(int variant) {
+  return variant == 2 ? (const void*)STM_SYM(stm_count_kernel_occ) : (const void*)STM_SYM(stm_count_kernel);
+}
+
+#if !STM_INSTR
 int stm_hash_compiled() { return STM_WITH_HASH; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
   return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);
 }
+#endif
 
-int stm_occupancy(int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm) {
+int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm) {
+  const void* fn = STM_SYM(kernel_fn)(variant);
   int smem = stm_smem_bytes(block_warps, k, n_nodes, ht_slots);
-  cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   // The DFS stacks are the only shared-memory users: carve out just enough shared
   // memory for the register-limited number of resident blocks and leave the rest
   // of the unified 256 KB array to L1, which caches the binary-search probes.
   cudaFuncAttributes fa;
-  e = cudaFuncGetAttributes(&fa, stm_count_kernel);
+  e = cudaFuncGetAttributes(&fa, fn);
   if (e != cudaSuccess) return (int)e;
   const int threads = block_warps * 32;
   const int regs_per_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
@@ -1459,20 +1598,21 @@ int stm_occupancy(int block_warps, int k, int n_nodes, int ht_slots, int* blocks
   pct = std::max(0, std::min(100, pct));
   if (const char* cv = getenv("STM_CARVEOUT")) pct = atoi(cv);  // experiments: -1 = leave the driver default
   if (pct >= 0) {
-    e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
     if (e != cudaSuccess) return (int)e;
   }
   (void)threads;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, stm_count_kernel, block_warps * 32, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, block_warps * 32, smem);
   return (int)e;
 }
 
-int stm_launch(const StmKParams& kp, int grid, void* stream) {
+int STM_SYM(stm_launch)(int variant, const StmKParams& kp, int grid, void* stream) {
+  const void* fn = STM_SYM(kernel_fn)(variant);
   int smem = stm_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes, kp.ht_slots);
-  cudaError_t e = cudaFuncSetAttribute(stm_count_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   void* args[] = {(void*)&kp};
-  e = cudaLaunchCooperativeKernel((const void*)stm_count_kernel, dim3(grid), dim3(kp.block_warps * 32), args,
+  e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kp.block_warps * 32), args,
                                   (size_t)smem, (cudaStream_t)stream);
   return (int)e;
 }

@@ -53,6 +53,7 @@ struct StmKParams {
   // Hub adjacency bitmaps: hub_slot[v] >= 0 selects the
   // n-bit row bitmaps[slot * bm_words ...] of N(v); membership probes into such a
   // row read one word instead of a binary search.  hub_slot == NULL: none.
+  const int32_t* out_start;       // [n]: index in N(v) of the first neighbour > v (NULL: none)
   const int32_t* hub_slot;
   const uint32_t* bitmaps;
   int64_t bm_words;
@@ -79,7 +80,10 @@ struct StmKParams {
 int stm_hash_compiled();
 // size in bytes of the dynamic shared memory for one block
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
+// kernel variants (register budgets): 1 = 64 registers, 2 = 40 registers (more warps)
 // launches the persistent kernel (cooperative); returns cudaError_t as int
-int stm_launch(const StmKParams& kp, int grid, void* stream);
+int stm_launch(int variant, const StmKParams& kp, int grid, void* stream);
+int stm_launch_instr(int variant, const StmKParams& kp, int grid, void* stream);  // instrumented build
 // max co-resident blocks per SM for the given block size
-int stm_occupancy(int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
+int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
+int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);

@@ -19,7 +19,10 @@
 
 #define STM_KMAX 8
 #define STM_MAX_NODES 32
-#define STM_UMAX 16        // max siblings per unrolled frame (levels >= 2)
+#ifndef STM_UMAX
+#define STM_UMAX 32
+#endif
+// max siblings per unrolled frame (levels >= 2)
 #define STM_RMAX 32        // max root siblings in frame 1
 
 enum { STM_SRC_NODE = 0, STM_SRC_RAW = 1 };

@@ -74,6 +74,7 @@ struct stm_graph {
   bool owns_csr = true;
   std::vector<int32_t> label_values;  // dense id -> label value
   int num_sms = 0;
+  int l2_bytes = 0;
   // Degree-ranked copy: vertex i of
   // the copy is the i-th vertex in (degree, id) order.  Plans whose restrictions
   // are order-free (STM_AUTO_RESTRICT or none) count on it; the count is the same
@@ -83,6 +84,10 @@ struct stm_graph {
   int32_t* d_rcol_idx = nullptr;
   uint8_t* d_rlabels = nullptr;
   int32_t* d_rank2orig = nullptr;  // [n]: ranked id -> caller's id (per-root output)
+  // out_start[v] = index in N(v) of the first neighbour > v, per numbering (NULL if
+  // it could not be built; then the kernel narrows by binary search alone)
+  int32_t* d_out_start = nullptr;
+  int32_t* d_rout_start = nullptr;
   // Hub adjacency bitmaps, per numbering ([0] caller's ids, [1] degree-ranked),
   // built lazily by the first launch that asks for them.
   struct HubBitmaps {
@@ -194,6 +199,34 @@ static void build_ranked(stm_graph* g) {
   g->d_rrow_ptr = nullptr;
   g->d_rcol_idx = nullptr;
   g->d_rlabels = nullptr;
+}
+
+// ---------------------------------------------------------------- out_start
+__global__ void out_start_fill(const int64_t* rp, const int32_t* ci, int64_t n, int32_t* out) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    int64_t lo = rp[v], hi = rp[v + 1];
+    const int64_t b = lo;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (ci[mid] <= v) lo = mid + 1; else hi = mid;
+    }
+    out[v] = (int32_t)(lo - b);
+  }
+}
+
+static int32_t* build_out_start(const int64_t* rp, const int32_t* ci, int64_t n) {
+  int32_t* d = nullptr;
+  if (n < 1 || cudaMalloc(&d, sizeof(int32_t) * n) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  out_start_fill<<<(unsigned)std::min<int64_t>((n + 255) / 256, 8192), 256>>>(rp, ci, n, d);
+  if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
+    cudaGetLastError();
+    cudaFree(d);
+    return nullptr;
+  }
+  return d;
 }
 
 // ---------------------------------------------------------------- hub bitmaps
@@ -361,12 +394,15 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
   if (e == cudaSuccess && nnz) e = cudaMemcpy(g->d_col_idx, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice);
   if (e == cudaSuccess && labels && n) e = cudaMemcpy(g->d_labels, dense.data(), n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, device);
   if (e != cudaSuccess) {
     stm_graph_free(g);
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
                     cudaGetErrorString(e));
   }
   build_ranked(g);
+  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
+  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
   *out = g;
   return STM_OK;
 }
@@ -422,7 +458,10 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
     }
   }
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
+  cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, device);
   build_ranked(g);
+  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
+  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
   *out = g;
   return STM_OK;
 }
@@ -451,6 +490,8 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
   cudaFree(g->d_rrow_ptr);
   cudaFree(g->d_rcol_idx);
   cudaFree(g->d_rlabels);
+  cudaFree(g->d_out_start);
+  cudaFree(g->d_rout_start);
   free_hub(g->hub[0]);
   free_hub(g->hub[1]);
   delete g;
@@ -464,7 +505,8 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->global_steal = 1;
   t->stop_level = 2;
   t->detect_level = 2;
-  t->unroll = 8;
+  t->unroll = 0;      // auto: 32 with the 40-register kernel, 16 with the 64-register one (measured)
+  t->occupancy = 0;   // auto: 40-register kernel when the CSR does not fit in half the L2
   t->root_chunk = 2;  // measured on B200 (tools/gpu_tune.sh): 32 -> 2 is 1.5-1.8x on C2/C3, neutral on C5
   t->block_warps = 16;
   t->blocks_per_sm = 0;
@@ -480,7 +522,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   stm_graph* g = const_cast<stm_graph*>(gc);
   stm_tuning t;
   if (tin) t = *tin; else stm_tuning_default(&t);
-  if (t.unroll < 1 || t.unroll > STM_UMAX) return stm_fail(STM_EINVAL, "unroll %d not in 1..%d", t.unroll, STM_UMAX);
+  if (t.unroll < 0 || t.unroll > STM_UMAX) return stm_fail(STM_EINVAL, "unroll %d not in 0..%d", t.unroll, STM_UMAX);
+  if (t.occupancy < 0 || t.occupancy > 2) return stm_fail(STM_EINVAL, "occupancy %d not in 0..2", t.occupancy);
   if (t.root_chunk < 1) return stm_fail(STM_EINVAL, "root_chunk %d < 1", t.root_chunk);
   if (t.block_warps == 0) t.block_warps = 16;
   if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
@@ -507,6 +550,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.col_idx = use_rank ? g->d_rcol_idx : g->d_col_idx;
   kp.labels = use_rank ? g->d_rlabels : g->d_labels;
   kp.root_map = use_rank ? g->d_rank2orig : nullptr;
+  kp.out_start = t.narrow_split == 0 ? (use_rank ? g->d_rout_start : g->d_out_start) : nullptr;
   kp.n = g->n;
   {
     const int min_deg = t.bitmap_min_degree == 0 ? STM_BITMAP_AUTO_MIN_DEGREE : t.bitmap_min_degree;
@@ -530,7 +574,13 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.global_steal = t.global_steal;
   kp.stop_level = t.stop_level;
   kp.detect_level = t.detect_level;
-  kp.unroll = t.unroll;
+  // kernel variant: DRAM-resident graphs are latency-bound -> more warps
+  int variant = t.occupancy;
+  if (variant == 0) {
+    const int64_t csr = (int64_t)g->nnz * 4 + (g->n + 1) * 8;
+    variant = csr > (int64_t)g->l2_bytes / 2 ? 2 : 1;
+  }
+  kp.unroll = t.unroll ? t.unroll : (variant == 2 ? 32 : 16);
   kp.root_batch = std::max(1, std::min(STM_RMAX, t.root_chunk));
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
@@ -545,7 +595,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
 
   int bps = 0;
-  int oe = stm_occupancy(t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
+  int oe = (t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy: %s", cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -597,7 +647,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   cudaStream_t st = (cudaStream_t)stream;
   CU(cudaMemsetAsync(S->state, 0, state_bytes, st));
-  int le = stm_launch(kp, grid, stream);
+  int le = (t.instrument ? stm_launch_instr : stm_launch)(variant, kp, grid, stream);
   if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
   g_info.grid = grid;
   g_info.block_threads = t.block_warps * 32;
@@ -605,6 +655,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   g_info.arena_bytes = (int64_t)arena_bytes;
   g_info.cap = kp.cap;
   g_info.ranked = use_rank ? 1 : 0;
+  g_info.variant = variant;
+  g_info.unroll = kp.unroll;
   if (d_count_out) {
     CU(cudaMemcpyAsync(d_count_out, &work->count, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
   }

@@ -34,7 +34,7 @@ class stm_tuning(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("local_steal", "global_steal", "stop_level", "detect_level",
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
                                                "instrument", "hash_slots", "vertex_order",
-                                               "bitmap_min_degree", "bitmap_budget_mb")]
+                                               "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "narrow_split")]
 
 
 class stm_shard(ctypes.Structure):
@@ -48,7 +48,7 @@ class stm_launch_info(ctypes.Structure):
                 ("global_steals", ctypes.c_int64), ("chunks", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("merge_bytes", ctypes.c_int64), ("jobs", ctypes.c_int64), ("ranked", ctypes.c_int32),
                 ("reserved", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64),
-                ("hubs", ctypes.c_int64)]
+                ("hubs", ctypes.c_int64), ("variant", ctypes.c_int32), ("unroll", ctypes.c_int32)]
 
 
 def _load():

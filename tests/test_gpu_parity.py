@@ -123,6 +123,9 @@ TUNINGS = [
     dict(root_chunk=32), dict(root_chunk=7, unroll=3),
     dict(bitmap_min_degree=1), dict(bitmap_min_degree=-1), dict(bitmap_min_degree=1, vertex_order=1),
     dict(bitmap_min_degree=40, unroll=1),
+    dict(narrow_split=1), dict(narrow_split=1, vertex_order=1, bitmap_min_degree=-1),
+    dict(occupancy=2), dict(occupancy=2, unroll=32, vertex_order=1), dict(occupancy=1, unroll=32),
+    dict(occupancy=2, unroll=5, root_chunk=1, stop_level=3, detect_level=3),
 ]
 
 
