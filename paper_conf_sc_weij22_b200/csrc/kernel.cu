@@ -152,6 +152,7 @@ __device__ __forceinline__ int bcast(int x) { return __shfl_sync(FULLMASK, x, 0)
 __device__ __forceinline__ int lbound(const int* __restrict__ a, int n, int x) {
   if (n <= 0) return 0;
   const int* base = a;
+#pragma unroll 1
   while (n > 1) {
     const int half = n >> 1;
     base = (base[half] < x) ? base + half : base;
@@ -163,6 +164,7 @@ __device__ __forceinline__ int lbound(const int* __restrict__ a, int n, int x) {
 __device__ __forceinline__ bool member(const int* __restrict__ a, int n, int x) {
   if (n <= 0) return false;
   const int* base = a;
+#pragma unroll 1
   while (n > 1) {
     const int half = n >> 1;
     base = (base[half] <= x) ? base + half : base;
