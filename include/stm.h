@@ -61,7 +61,11 @@ enum {
   STM_VERTEX_INDUCED = 1,  /* pattern non-edges must be data non-edges: set differences */
   STM_NO_CODE_MOTION = 2,  /* recompute every level's candidate set from raw neighbour lists (ablation) */
   STM_AUTO_RESTRICT = 4,   /* ignore `restr`; use Grochow-Kellis symmetry-breaking restrictions */
-  STM_AUTO_ORDER = 8       /* ignore `order`; use the greedy connected order */
+  STM_AUTO_ORDER = 8,      /* ignore `order`; use the greedy connected order */
+  STM_LAZY_UNBOUNDED = 16  /* code motion hoists only set chains that carry a restriction bound for their
+                              consumer; a chain unbounded at its first operation is computed at the level
+                              of its first consumer (no hoisting across levels whose prefixes rarely extend;
+                              speed only) */
 };
 
 enum { STM_K_MAX = 8 };

@@ -116,9 +116,10 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   if (k < 2) return stm_fail(STM_EINVAL, "pattern size k=%d < 2 is not a matching query", k);
   if (k > STM_KMAX) return stm_fail(STM_EUNSUPPORTED, "pattern size k=%d > %d", k, STM_KMAX);
   if (n_edges < 1 || !edges) return stm_fail(STM_EINVAL, "pattern has no edges");
-  if (flags & ~0xFu) return stm_fail(STM_EINVAL, "unknown flag bits 0x%x", flags);
+  if (flags & ~0x1Fu) return stm_fail(STM_EINVAL, "unknown flag bits 0x%x", flags);
   const bool vi = flags & STM_VERTEX_INDUCED;
   const bool cm = !(flags & STM_NO_CODE_MOTION);
+  const bool lazy = cm && (flags & STM_LAZY_UNBOUNDED);
 
   int adj[STM_KMAX][STM_KMAX] = {};
   std::vector<std::pair<int, int>> E;
@@ -328,13 +329,24 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     std::vector<int> key = {c.f};
     if (!cm) key.push_back(100 + l);  // no sharing across targets without code motion
     int prev_kind = STM_SRC_RAW, prev = c.f;
+    int lazy_level = 0;  // lazy mode: once a chain op is unbounded for this consumer, it and the
+                         // rest of the chain are computed at the consumer's level
     for (size_t t = 0; t < c.ops.size(); ++t) {
       key.push_back(c.ops[t].first * 16 + c.ops[t].second);
+      int level = c.level[t];
+      if (lazy) {
+        const unsigned known = (1u << c.level[t]) - 1;
+        const unsigned lo = reduce_lo(lo_pos[l] & known), hi = reduce_hi(hi_pos[l] & known);
+        if (!lo && !hi && !lazy_level) lazy_level = l;
+        if (lazy_level) level = lazy_level;
+        if (prev_kind == STM_SRC_NODE) level = std::max(level, tn[prev].level);
+        key.push_back(1000 + (int)(lo | hi << 8));  // no sharing across bound classes
+      }
       auto it = key2node.find(key);
       int id;
       if (it == key2node.end()) {
         id = (int)tn.size();
-        tn.push_back({c.level[t], prev_kind, prev, c.ops[t].second, c.ops[t].first, {}});
+        tn.push_back({level, prev_kind, prev, c.ops[t].second, c.ops[t].first, {}});
         key2node[key] = id;
       } else {
         id = it->second;

@@ -16,6 +16,7 @@ LIB_PATH = os.environ.get("STM_LIB_PATH") or os.path.join(_HERE, "libstm.so")  #
 
 STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW = range(6)
 STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
+STM_LAZY_UNBOUNDED = 16
 _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW"}
 
 EXPORTS = ["stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
@@ -258,12 +259,13 @@ class Plan:
     """Compiled pattern (owns the stm_plan handle)."""
 
     def __init__(self, k: int, edges, labels=None, order=None, restrictions=None, vertex_induced=False,
-                 code_motion=True, auto_restrict=None, auto_order=False):
+                 code_motion=True, auto_restrict=None, auto_order=False, lazy_unbounded=False):
         if auto_restrict is None:
             auto_restrict = restrictions is None
         flags = (STM_VERTEX_INDUCED if vertex_induced else 0) | (0 if code_motion else STM_NO_CODE_MOTION)
         flags |= STM_AUTO_RESTRICT if auto_restrict else 0
         flags |= STM_AUTO_ORDER if auto_order else 0
+        flags |= STM_LAZY_UNBOUNDED if lazy_unbounded else 0
         self.handle = stm_pattern_compile(k, edges, labels, order, restrictions, flags)
         self.k, self.n_sets, self.aut = stm_plan_info(self.handle)
         self.first_vertex = stm_plan_first_vertex(self.handle)

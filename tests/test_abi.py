@@ -173,3 +173,20 @@ def test_no_code_motion_keeps_all_work_at_the_consumer_level(stm):
         m = re.match(r"S\d+: level (\d) .*= (\S+) ", x)
         if m:  # without code motion a set is only built at the level that consumes it
             assert int(m.group(1)) >= 2
+
+
+def test_lazy_unbounded_plan_k6_minus_e(stm):
+    """STM_LAZY_UNBOUNDED: the bounded chain that enumerates the K4 (v0 < v1 < v2 < v3)
+    stays hoisted; the unbounded common neighbourhood of the K4, needed only by the two
+    last pattern vertices, is built at level 4 as one staged chain and shared by both."""
+    p = CATALOG["k6_minus_e"]
+    _, lines = _plan_lines(stm, p.k, p.edges, lazy_unbounded=True)
+    sets = [_strip(x) for x in lines if x.startswith("S")]
+    assert sets == ["S0: level 2 stage 0 = N(v0) & N(v1)", "S1: level 3 stage 0 = S0 & N(v2)",
+                    "S2: level 4 stage 0 = N(v0) & N(v1)", "S3: level 4 stage 1 = S2 & N(v2)",
+                    "S4: level 4 stage 2 = S3 & N(v3)"]
+    assert any(x.startswith("S0:") and "lo={v1}" in x for x in lines)
+    assert any(x.startswith("cand 4: S4") for x in lines) and any(x.startswith("count 5: S4") for x in lines)
+    # cliques are bounded at every level: lazy changes nothing
+    k5 = CATALOG["k5"]
+    assert _plan_lines(stm, k5.k, k5.edges, lazy_unbounded=True)[1][2:] == _plan_lines(stm, k5.k, k5.edges)[1][2:]

@@ -261,3 +261,19 @@ def test_per_root_histogram(rmat_small):
                                    root_u=plan.first_vertex, per_root=True)
         assert tot2 == otot2 == otot
         assert np.array_equal(pr2[rank2orig], opr2)
+
+
+@pytest.mark.parametrize("name", SMALL + BIG)
+@pytest.mark.parametrize("vi", [False, True])
+def test_lazy_unbounded_code_motion(rmat_small, name, vi):
+    """STM_LAZY_UNBOUNDED (bound-split code motion) changes where sets are computed,
+    never the count: labeled and unlabeled, both vertex numberings."""
+    g, G = rmat_small
+    p = CATALOG[name]
+    want = ocount(g, p, vi)
+    assert gcount(G, p, vi, lazy_unbounded=True) == want, (name, vi)
+    t = stm.stm_tuning_default(vertex_order=1, unroll=3)
+    assert gcount(G, p, vi, tuning=t, lazy_unbounded=True) == want, (name, vi)
+    if p.k <= 6:
+        pl = tuple(int(x) for x in np.random.default_rng(p.k + 1).integers(0, 4, p.k))
+        assert gcount(G, p, vi, pl, lazy_unbounded=True) == ocount(g, p, vi, pl)

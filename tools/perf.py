@@ -12,13 +12,14 @@ for spec in specs:
     cfg, name = spec.split(":")[:2]
     vi = ":vi" in spec
     nocm = ":nocm" in spec
+    lazy = ":lazy" in spec
     if cfg not in graphs:
         g = stmgen.config_graph(cfg)
         graphs[cfg] = (g, stm.Graph.from_stmgen(g))
     g, G = graphs[cfg]
     p = stmgen.CATALOG[name]
     lab = stmgen.pattern_labels(p.k, 8, 7) if g.labels is not None else None
-    plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, code_motion=not nocm)
+    plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, code_motion=not nocm, lazy_unbounded=lazy)
     t = stm.stm_tuning_default(**{k: int(v) for k, v in tk.items()})
     best = 1e9
     try:
