@@ -351,7 +351,8 @@ def main():
             "gpu_launches": args.steps * len(plans),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
-                         "kernel": f"stm_count_kernel ({queries[dom][0]} launch)",
+                         "kernel": ("stm_count_kernel_occ" if info.get("variant") == 2 else "stm_count_kernel")
+                                   + f" ({queries[dom][0]} launch, unroll {info.get('unroll')})",
                          "algorithmic_bytes_per_launch": alg[dom], "algorithmic_bytes_per_step": W_step,
                          "peak_source": peak_src,
                          "note": "achieved = SURVEY.md 8(d) W of the dominant launch (instrumented launch) / "

@@ -166,6 +166,9 @@ typedef struct stm_tuning {
   int32_t occupancy;      /* kernel register budget: 1 = 64 registers (32 warps/SM), 2 = 40 registers
                              (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
                              than half the L2.  Speed only.  Default 0. */
+  int32_t root_order;     /* order in which root chunks are handed out: 1 = ascending vertex id,
+                             2 = descending; 0 = auto (descending on the degree-ranked copy, where the
+                             heavy roots have the high ids: longest work first).  Speed only. */
   int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
                              out_start[v] (first neighbour > v, built at load); 1 = binary search only.
                              Speed only.  Default 0. */

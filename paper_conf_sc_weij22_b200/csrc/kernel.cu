@@ -1007,6 +1007,11 @@ __device__ __noinline__ bool try_chunk(W& w) {
       if (rb < kp.n) {
         b = (int)rb;
         e = (int)min((long long)kp.n, rb + kp.chunk);
+        if (kp.root_desc) {  // chunk c covers [n - e, n - b): the highest ids first
+          const int nb = (int)(kp.n - e);
+          e = (int)(kp.n - b);
+          b = nb;
+        }
       } else {
         w.exhausted |= 1u << r;
       }

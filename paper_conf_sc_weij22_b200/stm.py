@@ -35,7 +35,8 @@ class stm_tuning(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in ("local_steal", "global_steal", "stop_level", "detect_level",
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
                                                "instrument", "hash_slots", "vertex_order",
-                                               "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "narrow_split")]
+                                               "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
+                                               "narrow_split")]
 
 
 class stm_shard(ctypes.Structure):

@@ -126,6 +126,7 @@ TUNINGS = [
     dict(narrow_split=1), dict(narrow_split=1, vertex_order=1, bitmap_min_degree=-1),
     dict(occupancy=2), dict(occupancy=2, unroll=32, vertex_order=1), dict(occupancy=1, unroll=32),
     dict(occupancy=2, unroll=5, root_chunk=1, stop_level=3, detect_level=3),
+    dict(root_order=1), dict(root_order=2, vertex_order=1), dict(root_order=2, root_chunk=3, occupancy=2),
 ]
 
 
