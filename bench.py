@@ -307,12 +307,14 @@ def main():
     dom = max(range(len(plans)), key=lambda i: avg_launch_s[i])
     W_step = float(sum(alg))
     achieved = alg[dom] / avg_launch_s[dom] / 1e9
-    traffic, traffic_src = None, None
+    traffic, traffic_src, ncu_ev = None, None, None
     prof = os.path.join(ROOT, "profiles", f"ncu_traffic_{args.workload}_{queries[dom][0]}.json")
     if os.path.exists(prof):
         try:
             pj = _json.load(open(prof))
             traffic, traffic_src = pj.get("dram_bytes_per_launch"), os.path.relpath(prof, ROOT)
+            ncu_ev = {k: pj[k] for k in ("warp_execution_efficiency", "dram_read_gbs", "l2_gbs", "l1_hit_pct",
+                                         "l2_hit_pct", "warps_active_pct") if k in pj}
         except Exception:
             traffic = None
 
@@ -351,6 +353,7 @@ def main():
             "gpu_launches": args.steps * len(plans),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                         "ncu": ncu_ev,
                          "kernel": ("stm_count_kernel_occ" if info.get("variant") == 2 else "stm_count_kernel")
                                    + f" ({queries[dom][0]} launch, unroll {info.get('unroll')})",
                          "algorithmic_bytes_per_launch": alg[dom], "algorithmic_bytes_per_step": W_step,

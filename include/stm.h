@@ -145,7 +145,8 @@ typedef struct stm_tuning {
   int32_t detect_level;   /* donors look for idle blocks at frames < detect_level (paper: 1). Default 2. */
   int32_t unroll;         /* sibling iterations expanded together, 1..32 (paper: 8);
                              0 = auto (32 with the 40-register kernel, else 16; measured).  Default 0. */
-  int32_t root_chunk;     /* roots per cursor grab, 1..32. Default 2 (measured best on B200). */
+  int32_t root_chunk;     /* roots per cursor grab, 1..32; 0 = auto (1 with the 64-register kernel,
+                             2 with the 40-register one; measured on B200).  Default 0. */
   int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
   int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
@@ -167,8 +168,8 @@ typedef struct stm_tuning {
                              (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
                              than half the L2.  Speed only.  Default 0. */
   int32_t root_order;     /* order in which root chunks are handed out: 1 = ascending vertex id,
-                             2 = descending; 0 = auto (descending on the degree-ranked copy, where the
-                             heavy roots have the high ids: longest work first).  Speed only. */
+                             2 = descending (heavy roots first on the degree-ranked copy); 0 = auto
+                             (ascending: descending measured slower on C2/C3).  Speed only. */
   int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
                              out_start[v] (first neighbour > v, built at load); 1 = binary search only.
                              Speed only.  Default 0. */
@@ -187,7 +188,7 @@ void stm_tuning_default(stm_tuning* t);
  */
 typedef struct stm_shard {
   int32_t rank, world;           /* 0 <= rank < world <= 8 */
-  int32_t chunk;                 /* roots per chunk (>= 1) */
+  int32_t chunk;                 /* roots per chunk (>= 1); 0 = the launch's automatic root_chunk */
   int32_t reserved;
   uint64_t* d_cursors[8];        /* d_cursors[r] = device pointer to rank r's cursor (own entry
                                     required; peers NULL = no cross-GPU stealing).  The caller zeroes

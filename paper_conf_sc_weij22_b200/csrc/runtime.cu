@@ -508,7 +508,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->unroll = 0;      // auto: 32 with the 40-register kernel, 16 with the 64-register one (measured)
   t->occupancy = 0;   // auto: 40-register kernel when the CSR does not fit in half the L2
   t->root_order = 0;  // auto
-  t->root_chunk = 2;  // measured on B200 (tools/gpu_tune.sh): 32 -> 2 is 1.5-1.8x on C2/C3, neutral on C5
+  t->root_chunk = 0;  // auto: 1 with the 64-register kernel, 2 with the 40-register one (measured)
   t->block_warps = 16;
   t->blocks_per_sm = 0;
   t->bitmap_min_degree = 0;  // auto
@@ -526,7 +526,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.unroll < 0 || t.unroll > STM_UMAX) return stm_fail(STM_EINVAL, "unroll %d not in 0..%d", t.unroll, STM_UMAX);
   if (t.occupancy < 0 || t.occupancy > 2) return stm_fail(STM_EINVAL, "occupancy %d not in 0..2", t.occupancy);
   if (t.root_order < 0 || t.root_order > 2) return stm_fail(STM_EINVAL, "root_order %d not in 0..2", t.root_order);
-  if (t.root_chunk < 1) return stm_fail(STM_EINVAL, "root_chunk %d < 1", t.root_chunk);
+  if (t.root_chunk < 0) return stm_fail(STM_EINVAL, "root_chunk %d < 0", t.root_chunk);
   if (t.block_warps == 0) t.block_warps = 16;
   if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
   if (t.stop_level < 1) t.stop_level = 1;
@@ -538,7 +538,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   if (shard) {
     if (shard->world < 1 || shard->world > 8 || shard->rank < 0 || shard->rank >= shard->world ||
-        shard->chunk < 1 || !shard->d_cursors[shard->rank])
+        shard->chunk < 0 || !shard->d_cursors[shard->rank])
       return stm_fail(STM_EINVAL, "bad shard");
   }
   DeviceGuard dg(g->device);
@@ -583,10 +583,11 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     variant = csr > (int64_t)g->l2_bytes / 2 ? 2 : 1;
   }
   kp.unroll = t.unroll ? t.unroll : (variant == 2 ? 32 : 16);
-  // root order: on the degree-ranked copy the heavy roots sit at the high ids; taking
-  // them first (longest work first) shortens the tail (auto = descending when ranked)
-  kp.root_desc = t.root_order == 0 ? (use_rank ? 1 : 0) : (t.root_order == 2 ? 1 : 0);
-  kp.root_batch = std::max(1, std::min(STM_RMAX, t.root_chunk));
+  const int root_chunk = t.root_chunk ? t.root_chunk : (variant == 2 ? 2 : 1);
+  // root order: ascending by default -- descending (high-degree roots first on the
+  // ranked copy) measured 1.2-1.7x slower on C2/C3 and neutral on C5
+  kp.root_desc = t.root_order == 2 ? 1 : 0;
+  kp.root_batch = std::max(1, std::min(STM_RMAX, root_chunk));
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
     return stm_fail(STM_EINVAL, "hash_slots %d: 0 or a power of two in 64..4096", t.hash_slots);
@@ -642,12 +643,12 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (shard) {
     kp.rank = shard->rank;
     kp.world = shard->world;
-    kp.chunk = shard->chunk;
+    kp.chunk = shard->chunk ? shard->chunk : root_chunk;
     for (int r = 0; r < shard->world; ++r) kp.cursors[r] = (unsigned long long*)shard->d_cursors[r];
   } else {
     kp.rank = 0;
     kp.world = 1;
-    kp.chunk = t.root_chunk;
+    kp.chunk = root_chunk;
     kp.cursors[0] = own_cursor;
   }
   cudaStream_t st = (cudaStream_t)stream;

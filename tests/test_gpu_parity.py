@@ -278,3 +278,28 @@ def test_lazy_unbounded_code_motion(rmat_small, name, vi):
     if p.k <= 6:
         pl = tuple(int(x) for x in np.random.default_rng(p.k + 1).integers(0, 4, p.k))
         assert gcount(G, p, vi, pl, lazy_unbounded=True) == ocount(g, p, vi, pl)
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+@pytest.mark.parametrize("peers", [False, True])
+@pytest.mark.parametrize("chunk", [0, 3])
+def test_sharded_ranks_on_one_gpu(rmat_small, world, peers, chunk):
+    """The multi-GPU root partition through the C ABI: `world` ranks'
+    launches share one device's cursor array (peer pointers = the other ranks' cursors,
+    as torch symmetric memory maps them over NVLink).  Static partition (no peers) and
+    cross-rank stealing (peers: the first launch drains every cursor) both cover every
+    root chunk exactly once: the partial counts sum to the oracle's count."""
+    g, G = rmat_small
+    for name, vi in [("k4", False), ("house", True), ("c5", False)]:
+        p = CATALOG[name]
+        plan = stm.Plan(p.k, p.edges, vertex_induced=vi)
+        want = ocount(g, p, vi)
+        cur = torch.zeros(world * 8, dtype=torch.int64, device="cuda")
+        ptrs = [cur.data_ptr() + 64 * r for r in range(world)]
+        parts = []
+        for r in range(world):
+            sh = stm.make_shard(r, world, chunk, [ptrs[q] if (peers or q == r) else None for q in range(world)])
+            parts.append(stm.stm_match_count_ex(G.handle, plan.handle, None, sh, None))
+        assert sum(parts) % (1 << 64) == want, (name, world, peers, chunk, parts)
+        if peers:
+            assert parts[0] == want and all(x == 0 for x in parts[1:])

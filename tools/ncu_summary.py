@@ -15,7 +15,8 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_bytes.sum.per_second",
         "l1tex__t_bytes.sum.per_second", "dram__bytes_read.sum.per_second", "launch__registers_per_thread",
         "launch__grid_size", "launch__block_size", "sm__cycles_elapsed.avg.per_second",
-        "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active"]
+        "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "lts__t_sectors.sum",
+        "lts__t_sectors.sum.per_second"]
 
 
 def main(rep, out):
