@@ -229,6 +229,28 @@ stm_status stm_match_count_async(const stm_graph* g, const stm_plan* p, const st
 stm_status stm_match_count_per_root(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
                                     void* cuda_stream, uint64_t* per_root, uint64_t* count);
 
+/*
+ * stm_match_list -- enumerate the embeddings (PAPER.md:75 and :99,
+ * Output(C, iter) at the last level of the stack loop) instead of only counting them.
+ *   root_begin, root_end  the page of the root space to enumerate: embeddings whose
+ *                 level-0 vertex has counting id in [root_begin, root_end); [0, n)
+ *                 enumerates everything.  Counting ids are the caller's vertex ids, or
+ *                 (stm_tuning.vertex_order == 0 with order-free restrictions) positions in
+ *                 (degree, id) order; pages of any partition of [0, n) enumerate every
+ *                 embedding exactly once.
+ *   out          HOST int32[capacity][k]: row i = (f(0), ..., f(k-1)) in pattern-vertex
+ *                 order, caller's vertex ids, rows in no particular order.  May be NULL
+ *                 when capacity == 0 (count only).
+ *   n_listed     receives min(count, capacity): rows written.
+ *   count        receives the number of embeddings of the page (mod 2^64).  When count >
+ *                 capacity the rows are an arbitrary subset: split the page and repeat.
+ * The device buffer (capacity * k * 4 bytes) is allocated and freed by the call.  Errors:
+ * STM_EINVAL (bad range, NULL out with capacity > 0), STM_ENOMEM, STM_ECUDA.
+ */
+stm_status stm_match_list(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                          int64_t root_begin, int64_t root_end, void* cuda_stream, int32_t* out,
+                          uint64_t capacity, uint64_t* n_listed, uint64_t* count);
+
 /* stm_plan_first_vertex -- the pattern vertex matched at level 0 (order[0]). */
 stm_status stm_plan_first_vertex(const stm_plan* p, int* u0);
 

@@ -50,7 +50,8 @@ def build() -> str:
 def _load():
     global _lib
     if _lib is None:
-        if not os.path.exists(_LIB_PATH):
+        src = os.path.join(_HERE, "oracle.c")
+        if not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
             build()
         lib = ctypes.CDLL(_LIB_PATH)
         vp = ctypes.c_void_p
@@ -58,6 +59,11 @@ def _load():
         lib.oracle_count.argtypes = [ctypes.c_int64, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp, vp,
                                      ctypes.c_int, ctypes.c_int, vp, ctypes.c_int, vp, ctypes.c_int64,
                                      ctypes.c_int, vp, ctypes.POINTER(ctypes.c_uint64)]
+        lib.oracle_list.restype = ctypes.c_int
+        lib.oracle_list.argtypes = [ctypes.c_int64, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp, vp,
+                                    ctypes.c_int, ctypes.c_int, vp, ctypes.c_int, vp, ctypes.c_int64,
+                                    ctypes.c_int, vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
+                                    ctypes.POINTER(ctypes.c_uint64)]
         _lib = lib
     return _lib
 
@@ -109,6 +115,32 @@ def count(g, k: int, edges: Sequence[Tuple[int, int]], plabels: Optional[Sequenc
     return (int(out.value), pr) if per_root else int(out.value)
 
 
+def list_embeddings(g, k: int, edges: Sequence[Tuple[int, int]], plabels: Optional[Sequence[int]] = None,
+                    vertex_induced: bool = False, restrictions: Sequence[Tuple[int, int]] = (),
+                    threads: int = 0, capacity: Optional[int] = None) -> np.ndarray:
+    """Every embedding f of Q in g as the rows of an int32 [count, k] array (row = f(0..k-1),
+    in pattern-vertex order), sorted lexicographically (Output(C, iter) at the
+    last level).  Counts first to size the buffer unless ``capacity`` is given."""
+    lib = _load()
+    if capacity is None:
+        capacity = count(g, k, edges, plabels, vertex_induced, restrictions, threads=threads)
+    rp = np.ascontiguousarray(g.row_ptr, dtype=np.int64)
+    ci = np.ascontiguousarray(g.col_idx, dtype=np.int32)
+    lab = None if plabels is None else np.ascontiguousarray(g.labels, dtype=np.int32)
+    e = np.ascontiguousarray(np.asarray(edges, dtype=np.int32).reshape(-1, 2))
+    pl = None if plabels is None else np.ascontiguousarray(np.asarray(plabels, dtype=np.int32))
+    r = np.ascontiguousarray(np.asarray(restrictions, dtype=np.int32).reshape(-1, 2))
+    buf = np.zeros((max(int(capacity), 1), k), dtype=np.int32)
+    out, nl = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    rc = lib.oracle_list(g.n, _ptr(rp), _ptr(ci), _ptr(lab), k, e.shape[0], _ptr(e), _ptr(pl),
+                         int(vertex_induced), r.shape[0], _ptr(r), -1, None, 0, threads or (os.cpu_count() or 1),
+                         _ptr(buf), int(capacity), ctypes.byref(nl), ctypes.byref(out))
+    if rc != 0:
+        raise ValueError("oracle_list rejected its input")
+    got = buf[:min(int(nl.value), int(capacity))]
+    return got[np.lexsort(got.T[::-1])] if got.shape[0] else got
+
+
 # ---------------------------------------------------------------- brute force
 def _adj_sets(g):
     return [set(int(x) for x in g.col_idx[g.row_ptr[v]:g.row_ptr[v + 1]]) for v in range(g.n)]
@@ -132,6 +164,25 @@ def brute_force_count(g, k: int, edges, plabels=None, vertex_induced=False, rest
             continue
         c += 1
     return c % (1 << 64)
+
+
+def brute_force_list(g, k: int, edges, plabels=None, vertex_induced=False, restrictions=()) -> np.ndarray:
+    """brute_force_count's maps themselves, as a lexicographically sorted int32 [count, k] array."""
+    A = _adj_sets(g)
+    E = {(min(a, b), max(a, b)) for a, b in edges}
+    non_edges = [(a, b) for a in range(k) for b in range(a + 1, k) if (a, b) not in E]
+    rows = []
+    for f in itertools.permutations(range(g.n), k):
+        if any(f[b] not in A[f[a]] for a, b in E):
+            continue
+        if vertex_induced and any(f[b] in A[f[a]] for a, b in non_edges):
+            continue
+        if plabels is not None and any(int(g.labels[f[u]]) != int(plabels[u]) for u in range(k)):
+            continue
+        if any(not f[a] < f[b] for a, b in restrictions):
+            continue
+        rows.append(f)
+    return np.array(sorted(rows), dtype=np.int32).reshape(-1, k)
 
 
 # ---------------------------------------------------------------- symmetry

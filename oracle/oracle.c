@@ -62,6 +62,11 @@ typedef struct {
   atomic_llong next;
   int64_t chunk;
   uint64_t *per_root;      /* NULL or [n_roots] (indexed like roots) */
+  /* listing (PAPER.md:75 Output(C, iter)): every embedding f, as f[0..k-1] in pattern-vertex
+     order, is appended at an atomically taken index; only indices < list_cap are written */
+  int32_t *list;
+  uint64_t list_cap;
+  atomic_ullong list_n;
 } ojob;
 
 typedef struct {
@@ -109,6 +114,11 @@ static void rec(ostate *S, int l) {
   const ojob *J = S->J;
   if (l == J->k) {
     S->count += 1;
+    if (J->list) {
+      uint64_t i = atomic_fetch_add((atomic_ullong *)&J->list_n, 1);
+      if (i < J->list_cap)
+        for (int u = 0; u < J->k; ++u) J->list[i * (uint64_t)J->k + u] = (int32_t)S->f[u];
+    }
     return;
   }
   int u = J->order[l];
@@ -144,7 +154,7 @@ static void *worker(void *arg) {
       for (int x = 0; x < OMAX; ++x) S->f[x] = -1;
       if (consistent(S, 0, u0, v)) {
         S->f[u0] = v;
-        if (J->k == 1) S->count += 1; else rec(S, 1);
+        rec(S, 1);
         S->f[u0] = -1;
       }
       if (J->per_root) J->per_root[i] = S->count - before;
@@ -186,11 +196,11 @@ static int bfs_order(int k, int adj[OMAX][OMAX], int root_u, int *order) {
  * given data vertices (NULL = all); `per_root` (optional) receives the count
  * attributed to each root, i.e. to f(root_u).
  */
-int oracle_count(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int32_t *labels,
-                 int k, int n_edges, const int32_t *edges, const int32_t *plabels,
-                 int vertex_induced, int n_restr, const int32_t *restr, int root_u,
-                 const int64_t *roots, int64_t n_roots, int nthreads, uint64_t *per_root,
-                 uint64_t *out_count) {
+static int run(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int32_t *labels,
+               int k, int n_edges, const int32_t *edges, const int32_t *plabels,
+               int vertex_induced, int n_restr, const int32_t *restr, int root_u,
+               const int64_t *roots, int64_t n_roots, int nthreads, uint64_t *per_root,
+               int32_t *list, uint64_t list_cap, uint64_t *list_n, uint64_t *out_count) {
   if (k < 1 || k > OMAX) return -1;
   ojob *J = (ojob *)calloc(1, sizeof(ojob));
   J->n = n; J->row_ptr = row_ptr; J->col_idx = col_idx; J->labels = labels;
@@ -218,6 +228,9 @@ int oracle_count(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, cons
   atomic_init(&J->next, 0);
   J->chunk = 64;
   J->per_root = per_root;
+  J->list = list;
+  J->list_cap = list_cap;
+  atomic_init(&J->list_n, 0);
   if (nthreads < 1) nthreads = 1;
   if (nthreads > 256) nthreads = 256;
   pthread_t th[256];
@@ -232,7 +245,29 @@ int oracle_count(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, cons
     total += S[t].count;
   }
   free(S);
+  if (list_n) *list_n = atomic_load(&J->list_n);
   free(J);
   *out_count = total;
   return 0;
+}
+
+/* count (see run) */
+int oracle_count(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int32_t *labels,
+                 int k, int n_edges, const int32_t *edges, const int32_t *plabels,
+                 int vertex_induced, int n_restr, const int32_t *restr, int root_u,
+                 const int64_t *roots, int64_t n_roots, int nthreads, uint64_t *per_root,
+                 uint64_t *out_count) {
+  return run(n, row_ptr, col_idx, labels, k, n_edges, edges, plabels, vertex_induced, n_restr, restr, root_u,
+             roots, n_roots, nthreads, per_root, NULL, 0, NULL, out_count);
+}
+
+/* count and list: list[i*k + u] = f(u) for the first min(count, list_cap) embeddings found
+   (in no particular order); *list_n = count as well (the number of listing slots taken) */
+int oracle_list(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int32_t *labels,
+                int k, int n_edges, const int32_t *edges, const int32_t *plabels,
+                int vertex_induced, int n_restr, const int32_t *restr, int root_u,
+                const int64_t *roots, int64_t n_roots, int nthreads,
+                int32_t *list, uint64_t list_cap, uint64_t *list_n, uint64_t *out_count) {
+  return run(n, row_ptr, col_idx, labels, k, n_edges, edges, plabels, vertex_induced, n_restr, restr, root_u,
+             roots, n_roots, nthreads, NULL, list, list_cap, list_n, out_count);
 }

@@ -62,8 +62,13 @@
 #ifndef STM_INSTR
 #define STM_INSTR 0         // 1: the instrumented build (kernel_instr.cu): algorithmic-byte / idle counters
 #endif
+#ifndef STM_LIST
+#define STM_LIST 0          // 1: the listing build (kernel_list.cu): last level emits embeddings (NEXT-1)
+#endif
 #if STM_INSTR
 #define STM_SYM(x) x##_instr
+#elif STM_LIST
+#define STM_SYM(x) x##_list
 #else
 #define STM_SYM(x) x
 #endif
@@ -421,7 +426,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   unsigned long long jc = 0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
                            Oll = (unsigned long long)J.out;
-#if STM_ILP2
+#if STM_ILP2 && !STM_LIST
   // two 32-element slices per iteration: slice h covers elements e0 + 32h + lane
   for (int e0 = 0; e0 < total; e0 += 64) {
     int j[2], x[2], fjs[2];
@@ -521,6 +526,18 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       }
       if (keep && labj != STM_LAB_ANY) keep = (l2s[glabels[x]] & labj) != 0;
     }
+#if STM_LIST
+    // listing build: injectivity exclusions are applied per element (instead of the
+    // count correction below), then every kept element is one embedding
+    int uj = 0, cj = 0;
+    if (count_mode) {
+      uj = __shfl_sync(FULLMASK, J.u, j);
+      cj = __shfl_sync(FULLMASK, J.c, j);
+      if (keep && excl)
+        for (int t = 0; t < STM_KMAX; ++t)
+          if ((excl >> t & 1u) && x == pval(w, t, F, uj, cj)) keep = false;
+    }
+#endif
     const unsigned km = __ballot_sync(FULLMASK, keep);
     // lanes of my own job inside this chunk
     int a = start - e0, b = incl - e0;
@@ -530,6 +547,25 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
     if (mine && a < b) rmask = (b == 32 ? FULLMASK : ((1u << b) - 1)) & ~((1u << a) - 1);
     if (count_mode) {
       jc += __popc(km & rmask);
+#if STM_LIST
+      if (km) {
+        // PAPER.md:75 Output(C, iter): row = f(0..k-1) in pattern-vertex order, caller's ids
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(&w.kp->work->list_n, (unsigned long long)__popc(km));
+        base = __shfl_sync(FULLMASK, base, 0);
+        const unsigned long long idx = base + __popc(km & ((1u << lane) - 1));
+        if (keep && idx < w.kp->list_cap) {
+          const StmPlan& PL = *w.P;
+          int32_t* row = w.kp->list_out + idx * (unsigned long long)PL.k;
+          const int32_t* rmap = w.kp->root_map;
+          for (int t = 0; t < PL.k - 1; ++t) {
+            const int v = pval(w, t, F, uj, cj);
+            row[PL.order[t]] = rmap ? rmap[v] : v;
+          }
+          row[PL.order[PL.k - 1]] = rmap ? rmap[x] : x;
+        }
+      }
+#endif
     } else {
       int* Oj = (int*)__shfl_sync(FULLMASK, Oll, j);
       int base = __shfl_sync(FULLMASK, outc, j);
@@ -549,7 +585,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   }
   // exclusions: earlier matched vertices of non-adjacent pattern vertices may
   // still be in the counted set; remove them explicitly.
-  if (mine && excl) {
+  if (!STM_LIST && mine && excl) {
     for (int t = 0; t < STM_KMAX; ++t) {
       if (!(excl & (1u << t))) continue;
       int x = pval(w, t, F, J.u, J.c);
@@ -1003,13 +1039,13 @@ __device__ __noinline__ bool try_chunk(W& w) {
       if (!kp.cursors[r] || (w.exhausted & (1u << r))) continue;
       unsigned long long idx = atomicAdd(kp.cursors[r], 1ull);
       long long c = (long long)r + (long long)kp.world * (long long)idx;
-      long long rb = c * (long long)kp.chunk;
+      long long rb = kp.root_lo + c * (long long)kp.chunk;
       if (rb < kp.n) {
         b = (int)rb;
         e = (int)min((long long)kp.n, rb + kp.chunk);
-        if (kp.root_desc) {  // chunk c covers [n - e, n - b): the highest ids first
-          const int nb = (int)(kp.n - e);
-          e = (int)(kp.n - b);
+        if (kp.root_desc) {  // chunk c covers [lo + n - e, lo + n - b): the highest ids first
+          const int nb = (int)(kp.root_lo + kp.n - e);
+          e = (int)(kp.root_lo + kp.n - b);
           b = nb;
         }
       } else {
@@ -1577,7 +1613,7 @@ static const void* STM_SYM(kernel_fn)(int variant) {
   return variant == 2 ? (const void*)STM_SYM(stm_count_kernel_occ) : (const void*)STM_SYM(stm_count_kernel);
 }
 
-#if !STM_INSTR
+#if !STM_INSTR && !STM_LIST
 int stm_hash_compiled() { return STM_WITH_HASH; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {

@@ -34,6 +34,7 @@ struct StmWork {
   unsigned long long n_jobs;
   unsigned long long idle_cycles;  // sum over warps of cycles spent acquiring work (instrumented)
   unsigned long long warp_cycles;  // sum over warps of their lifetime in cycles (instrumented)
+  unsigned long long list_n;       // listing build: embeddings found (slots taken) so far
   unsigned long long prof[3 * STM_PROF_N + 4];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
                                                 // lifetime, max lifetime, summed / max time cursors ran dry
 };
@@ -57,7 +58,10 @@ struct StmKParams {
   const int32_t* hub_slot;
   const uint32_t* bitmaps;
   int64_t bm_words;
-  int64_t n;
+  int64_t n;                      // root space end: roots are [root_lo, n)
+  int64_t root_lo;
+  int32_t* list_out;              // listing build: [list_cap][k] rows (pattern-vertex order)
+  unsigned long long list_cap;
   int32_t cap;                    // words per set-node region per warp
   int32_t block_warps;
   int32_t* arena;                 // [total_warps][n_nodes][cap]
@@ -85,6 +89,8 @@ int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
 // launches the persistent kernel (cooperative); returns cudaError_t as int
 int stm_launch(int variant, const StmKParams& kp, int grid, void* stream);
 int stm_launch_instr(int variant, const StmKParams& kp, int grid, void* stream);  // instrumented build
+int stm_launch_list(int variant, const StmKParams& kp, int grid, void* stream);   // listing build
 // max co-resident blocks per SM for the given block size
 int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
 int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
+int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);

@@ -516,9 +516,16 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
 }
 
 // ---------------------------------------------------------------------------- match
+struct ListArgs {      // stm_match_list: root range and device output
+  int64_t root_lo = 0, root_hi = -1;
+  int32_t* d_out = nullptr;
+  uint64_t cap = 0;
+  uint64_t n_found = 0;  // out
+};
+
 static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tuning* tin,
                          const stm_shard* shard, void* stream, uint64_t* d_count_out,
-                         unsigned long long* d_per_root, uint64_t* h_count) {
+                         unsigned long long* d_per_root, uint64_t* h_count, ListArgs* la = nullptr) {
   if (!gc || !p) return stm_fail(STM_EINVAL, "NULL graph or plan");
   stm_graph* g = const_cast<stm_graph*>(gc);
   stm_tuning t;
@@ -554,6 +561,12 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.root_map = use_rank ? g->d_rank2orig : nullptr;
   kp.out_start = t.narrow_split == 0 ? (use_rank ? g->d_rout_start : g->d_out_start) : nullptr;
   kp.n = g->n;
+  if (la) {
+    kp.root_lo = la->root_lo;
+    kp.n = la->root_hi;
+    kp.list_out = la->d_out;
+    kp.list_cap = la->cap;
+  }
   {
     const int min_deg = t.bitmap_min_degree == 0 ? STM_BITMAP_AUTO_MIN_DEGREE : t.bitmap_min_degree;
     const int64_t budget = (int64_t)(t.bitmap_budget_mb > 0 ? t.bitmap_budget_mb : STM_BITMAP_AUTO_BUDGET_MB) << 20;
@@ -601,7 +614,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
 
   int bps = 0;
-  int oe = (t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
+  int oe = (la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy: %s", cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -653,7 +666,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   cudaStream_t st = (cudaStream_t)stream;
   CU(cudaMemsetAsync(S->state, 0, state_bytes, st));
-  int le = (t.instrument ? stm_launch_instr : stm_launch)(variant, kp, grid, stream);
+  int le = (la ? stm_launch_list : t.instrument ? stm_launch_instr : stm_launch)(variant, kp, grid, stream);
   if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
   g_info.grid = grid;
   g_info.block_threads = t.block_warps * 32;
@@ -681,6 +694,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     g_info.idle_cycles = (int64_t)hw.idle_cycles;
     memcpy(g_prof, hw.prof, sizeof g_prof);
     g_info.warp_cycles = (int64_t)hw.warp_cycles;
+    if (la) la->n_found = hw.list_n;
     *h_count = hw.count;
   }
   return STM_OK;
@@ -718,6 +732,41 @@ extern "C" stm_status stm_match_count_per_root(const stm_graph* g, const stm_pla
   }
   cudaFree(d);
   if (s == STM_OK) *count = c;
+  return s;
+}
+
+extern "C" stm_status stm_match_list(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
+                                     int64_t root_begin, int64_t root_end, void* stream, int32_t* out,
+                                     uint64_t capacity, uint64_t* n_listed, uint64_t* count) {
+  if (!g || !p || !n_listed || !count) return stm_fail(STM_EINVAL, "NULL argument");
+  if (capacity > 0 && !out) return stm_fail(STM_EINVAL, "out is NULL with capacity %llu", (unsigned long long)capacity);
+  if (root_begin < 0 || root_end < root_begin || root_end > g->n)
+    return stm_fail(STM_EINVAL, "root range [%lld, %lld) not within [0, %lld)", (long long)root_begin,
+                    (long long)root_end, (long long)g->n);
+  const int k = p->k;
+  if (capacity > (uint64_t)(INT64_MAX / 4 / k)) return stm_fail(STM_EINVAL, "capacity too large");
+  DeviceGuard dg(g->device);
+  int32_t* d = nullptr;
+  const size_t bytes = sizeof(int32_t) * (size_t)k * (size_t)std::max<uint64_t>(capacity, 1);
+  cudaError_t e = cudaMalloc(&d, bytes);
+  if (e != cudaSuccess) return stm_fail(STM_ENOMEM, "listing buffer of %zu bytes: %s", bytes, cudaGetErrorString(e));
+  ListArgs la;
+  la.root_lo = root_begin;
+  la.root_hi = root_end;
+  la.d_out = d;
+  la.cap = capacity;
+  uint64_t c = 0;
+  stm_status s = launch(g, p, t, nullptr, stream, nullptr, nullptr, &c, &la);
+  const uint64_t nl = std::min<uint64_t>(la.n_found, capacity);
+  if (s == STM_OK && nl) {
+    e = cudaMemcpy(out, d, sizeof(int32_t) * (size_t)k * (size_t)nl, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) s = stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+  }
+  cudaFree(d);
+  if (s == STM_OK) {
+    *n_listed = nl;
+    *count = c;
+  }
   return s;
 }
 

@@ -19,7 +19,7 @@ STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM
 STM_LAZY_UNBOUNDED = 16
 _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW"}
 
-EXPORTS = ["stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
+EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
            "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
            "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
            "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error"]
@@ -74,6 +74,8 @@ def _load():
         "stm_match_count_ex": [vp, vp, vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
         "stm_match_count_async": [vp, vp, vp, vp, vp, vp],
         "stm_match_count_per_root": [vp, vp, vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
+        "stm_match_list": [vp, vp, vp, i64, i64, vp, vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
+                           ctypes.POINTER(ctypes.c_uint64)],
         "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
     }
     for name, args in sig.items():
@@ -199,6 +201,21 @@ def stm_match_count_async(g: int, p: int, d_count: int, tuning: Optional[stm_tun
                           shard: Optional[stm_shard] = None, stream: Optional[int] = None) -> None:
     sp = None if shard is None else ctypes.cast(ctypes.pointer(shard), ctypes.c_void_p)
     _check(lib.stm_match_count_async(g, p, _tp(tuning), sp, stream, d_count))
+
+
+def stm_match_list(g: int, p: int, k: int, tuning: Optional[stm_tuning] = None, root_begin: int = 0,
+                   root_end: Optional[int] = None, capacity: int = 0, stream: Optional[int] = None):
+    """Enumerate embeddings of the root page [root_begin, root_end): returns (rows, count)
+    with rows an int32 [min(count, capacity), k] array (pattern-vertex order, caller's ids)."""
+    if root_end is None:
+        n = ctypes.c_int64()
+        _check(lib.stm_graph_info(g, ctypes.byref(n), None, None))
+        root_end = n.value
+    buf = np.zeros((max(capacity, 1), k), dtype=np.int32)
+    nl, c = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib.stm_match_list(g, p, _tp(tuning), root_begin, root_end, stream,
+                              buf.ctypes.data if capacity else None, capacity, ctypes.byref(nl), ctypes.byref(c)))
+    return buf[:nl.value], c.value
 
 
 def stm_match_count_per_root(g: int, p: int, tuning: Optional[stm_tuning] = None,

@@ -303,3 +303,73 @@ def test_sharded_ranks_on_one_gpu(rmat_small, world, peers, chunk):
         assert sum(parts) % (1 << 64) == want, (name, world, peers, chunk, parts)
         if peers:
             assert parts[0] == want and all(x == 0 for x in parts[1:])
+
+
+# ---------------------------------------------------------------- listing (NEXT-1)
+def _sorted_rows(a):
+    return a[np.lexsort(a.T[::-1])] if a.shape[0] else a
+
+
+def _canon(rows, aut):
+    """Orbit representative of every row: the lexicographically smallest automorphism image."""
+    if rows.shape[0] == 0:
+        return rows
+    imgs = np.stack([rows[:, [a.index(u) for u in range(rows.shape[1])]] for a in aut])  # [|Aut|, m, k]
+    best = imgs[0].copy()
+    for im in imgs[1:]:
+        for i in range(best.shape[0]):
+            if tuple(im[i]) < tuple(best[i]):
+                best[i] = im[i]
+    return _sorted_rows(best)
+
+
+@pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "house", "k4", "c5", "tailed_triangle", "path4"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_listing_matches_oracle(er_small, name, vi):
+    """stm_match_list rows (caller ids, pattern-vertex order) are exactly the oracle's
+    embeddings: caller numbering element by element; degree-ranked numbering (different
+    symmetry-breaking representatives of the same subgraphs) orbit by orbit."""
+    g, G = er_small
+    p = CATALOG[name]
+    R = oracle.gk_restrictions(p.k, p.edges)
+    want = oracle.list_embeddings(g, p.k, p.edges, vertex_induced=vi, restrictions=R)
+    plan = stm.Plan(p.k, p.edges, vertex_induced=vi)
+    rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, stm.stm_tuning_default(vertex_order=1),
+                                 capacity=want.shape[0] + 5)
+    assert c == want.shape[0] and np.array_equal(_sorted_rows(rows), want)
+    rows2, c2 = stm.stm_match_list(G.handle, plan.handle, p.k, None, capacity=want.shape[0] + 5)
+    assert stm.stm_last_launch()["ranked"] == 1
+    aut = oracle.automorphisms(p.k, p.edges)
+    assert c2 == c and np.array_equal(_canon(rows2, aut), _canon(want, aut))
+    # labeled and unrestricted
+    pl = tuple(int(x) for x in np.random.default_rng(p.k).integers(0, 3, p.k))
+    want3 = oracle.list_embeddings(g, p.k, p.edges, pl, vi)
+    plan3 = stm.Plan(p.k, p.edges, pl, restrictions=[], auto_restrict=False, vertex_induced=vi)
+    rows3, c3 = stm.stm_match_list(G.handle, plan3.handle, p.k, None, capacity=want3.shape[0])
+    assert c3 == want3.shape[0] and np.array_equal(_sorted_rows(rows3), want3)
+
+
+def test_listing_pages_and_capacity(rmat_small):
+    """Pages of the root space partition the embeddings; a short buffer returns a valid
+    subset and the full count (paging by splitting the root range)."""
+    g, G = rmat_small
+    p = CATALOG["diamond"]
+    R = oracle.gk_restrictions(p.k, p.edges)
+    want = oracle.list_embeddings(g, p.k, p.edges, restrictions=R)
+    plan = stm.Plan(p.k, p.edges)
+    t = stm.stm_tuning_default(vertex_order=1)
+    cuts = [0, 1, 100, 333, 334, 800, g.n]
+    parts, tot = [], 0
+    for b, e in zip(cuts[:-1], cuts[1:]):
+        rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, t, b, e, capacity=want.shape[0])
+        assert rows.shape[0] == c
+        if c:
+            assert np.all(rows[:, plan.first_vertex] >= b) and np.all(rows[:, plan.first_vertex] < e)
+        parts.append(rows)
+        tot += c
+    assert tot == want.shape[0] and np.array_equal(_sorted_rows(np.concatenate(parts)), want)
+    rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, t, capacity=7)
+    wanted = {tuple(r) for r in want}
+    assert c == want.shape[0] and rows.shape[0] == 7 and all(tuple(r) in wanted for r in rows)
+    rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, t, capacity=0)
+    assert c == want.shape[0] and rows.shape[0] == 0

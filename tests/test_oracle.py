@@ -266,3 +266,48 @@ def test_degenerate_inputs():
     assert ocount(stmgen.empty(0), p) == 0
     with pytest.raises(ValueError):
         oracle.count(stmgen.complete(4), 4, [(0, 1), (2, 3)])  # disconnected pattern
+
+
+# ------------------------------------------------------------------ listing (NEXT-1)
+@pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("mode", ["edge", "vertex"])
+def test_listing_equals_brute_force(seed, mode):
+    """Pin: the oracle's listing (PAPER.md:75 Output(C, iter)) is exactly the set of
+    maps that satisfy the definition, found by brute force over all injective maps."""
+    rng = np.random.default_rng(40 + seed)
+    n = 7
+    g = stmgen.er(n, int(rng.integers(9, 15)), 2000 + seed)
+    g.labels = stmgen.labels(n, 2, 88 + seed)
+    for name in ["triangle", "path4", "c4", "diamond", "house", "star4"]:
+        p = CATALOG[name]
+        pl = tuple(int(x) for x in rng.integers(0, 2, p.k))
+        for lab in (None, pl):
+            for R in ([], oracle.gk_restrictions(p.k, p.edges, lab)):
+                want = oracle.brute_force_list(g, p.k, p.edges, lab, mode == "vertex", R)
+                got = oracle.list_embeddings(g, p.k, p.edges, lab, mode == "vertex", R, threads=2)
+                assert np.array_equal(got, want), (name, mode, lab, R)
+
+
+def test_listing_orbits_cover_unrestricted():
+    """Invariant: the automorphism images of the restricted (distinct-subgraph) listing
+    are exactly the unrestricted listing, each embedding once (|Aut| * restricted =
+    unrestricted, element by element) -- on a graph too large for brute force."""
+    g = stmgen.er(60, 420, 31)
+    for name in ["c4", "diamond", "house", "k4", "c5"]:
+        p = CATALOG[name]
+        R = oracle.gk_restrictions(p.k, p.edges)
+        res = oracle.list_embeddings(g, p.k, p.edges, restrictions=R)
+        full = oracle.list_embeddings(g, p.k, p.edges)
+        aut = oracle.automorphisms(p.k, p.edges)
+        imgs = np.concatenate([res[:, [a.index(u) for u in range(p.k)]] for a in aut]) if res.size else res
+        imgs = imgs[np.lexsort(imgs.T[::-1])] if imgs.size else imgs
+        assert imgs.shape[0] == full.shape[0] == res.shape[0] * len(aut)
+        assert np.array_equal(imgs, full), name
+
+
+def test_listing_truncates_at_capacity():
+    g = stmgen.er(40, 200, 5)
+    p = CATALOG["triangle"]
+    full = oracle.list_embeddings(g, p.k, p.edges)
+    part = oracle.list_embeddings(g, p.k, p.edges, capacity=5)
+    assert part.shape == (5, 3) and all(tuple(r) in {tuple(x) for x in full} for r in part)
