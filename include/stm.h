@@ -170,6 +170,10 @@ typedef struct stm_tuning {
   int32_t root_order;     /* order in which root chunks are handed out: 1 = ascending vertex id,
                              2 = descending (heavy roots first on the degree-ranked copy); 0 = auto
                              (ascending: descending measured slower on C2/C3).  Speed only. */
+  int32_t l2_persist_mb;  /* L2 persisting access-policy window over the longest neighbour lists (the
+                             tail of the degree-ranked col_idx) when the CSR does not fit in half the L2:
+                             0 = auto (off: measured no gain on C5), -1 = off, else MiB (capped by the
+                             device; sets the device's persisting L2 limit).  Speed only. */
   int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
                              out_start[v] (first neighbour > v, built at load); 1 = binary search only.
                              Speed only.  Default 0. */

@@ -1655,7 +1655,28 @@ int STM_SYM(stm_launch)(int variant, const StmKParams& kp, int grid, void* strea
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   void* args[] = {(void*)&kp};
-  e = cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kp.block_warps * 32), args,
-                                  (size_t)smem, (cudaStream_t)stream);
+  // cooperative launch (co-residency for the spin-waiting scheduler) with an optional
+  // L2 access-policy window that keeps the hottest neighbour lists persisting in L2
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kp.block_warps * 32);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = (cudaStream_t)stream;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  int na = 1;
+  if (kp.l2_window_bytes > 0) {
+    at[1].id = cudaLaunchAttributeAccessPolicyWindow;
+    at[1].val.accessPolicyWindow.base_ptr = (void*)kp.l2_window_base;
+    at[1].val.accessPolicyWindow.num_bytes = (size_t)kp.l2_window_bytes;
+    at[1].val.accessPolicyWindow.hitRatio = 1.0f;
+    at[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    at[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    na = 2;
+  }
+  cfg.attrs = at;
+  cfg.numAttrs = na;
+  e = cudaLaunchKernelExC(&cfg, fn, args);
   return (int)e;
 }

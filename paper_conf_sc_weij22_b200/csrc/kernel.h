@@ -78,6 +78,8 @@ struct StmKParams {
   int32_t donate_mask;            // donors look for idle blocks every (mask+1)-th opportunity
   int32_t backoff_max;            // idle warps sleep up to 32 << backoff_max ns between steal attempts
   long long watchdog_cycles;      // debug: abort (set work->overflow = 2) after this many cycles; 0 = off
+  const void* l2_window_base;     // L2 persisting access-policy window (0 bytes = none)
+  long long l2_window_bytes;
   uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
 };
 

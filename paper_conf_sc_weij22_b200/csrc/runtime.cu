@@ -22,6 +22,7 @@
 // Hub bitmap defaults (stm_tuning 0 = auto): measured on B200, DESIGN.md "Hub bitmaps".
 #define STM_BITMAP_AUTO_MIN_DEGREE 64
 #define STM_BITMAP_AUTO_BUDGET_MB 2048
+#define STM_L2_PERSIST_AUTO_MB 0   // measured neutral at 24-48 MiB, worse at 96 MiB on C5: off
 
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
@@ -75,6 +76,8 @@ struct stm_graph {
   std::vector<int32_t> label_values;  // dense id -> label value
   int num_sms = 0;
   int l2_bytes = 0;
+  int64_t max_window = 0, persist_max = 0;  // cudaDevAttrMaxAccessPolicyWindowSize / MaxPersistingL2CacheSize
+  int64_t persist_set = 0;                  // persisting L2 set-aside this library last requested
   // Degree-ranked copy: vertex i of
   // the copy is the i-th vertex in (degree, id) order.  Plans whose restrictions
   // are order-free (STM_AUTO_RESTRICT or none) count on it; the count is the same
@@ -199,6 +202,15 @@ static void build_ranked(stm_graph* g) {
   g->d_rrow_ptr = nullptr;
   g->d_rcol_idx = nullptr;
   g->d_rlabels = nullptr;
+}
+
+static void query_persist(stm_graph* g) {
+  int a = 0, b = 0;
+  if (cudaDeviceGetAttribute(&a, cudaDevAttrMaxAccessPolicyWindowSize, g->device) != cudaSuccess) a = 0;
+  if (cudaDeviceGetAttribute(&b, cudaDevAttrMaxPersistingL2CacheSize, g->device) != cudaSuccess) b = 0;
+  cudaGetLastError();
+  g->max_window = a;
+  g->persist_max = b;
 }
 
 // ---------------------------------------------------------------- out_start
@@ -395,6 +407,7 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
   if (e == cudaSuccess && labels && n) e = cudaMemcpy(g->d_labels, dense.data(), n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, device);
+  query_persist(g);
   if (e != cudaSuccess) {
     stm_graph_free(g);
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
@@ -459,6 +472,7 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
   }
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
   cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, device);
+  query_persist(g);
   build_ranked(g);
   g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
   if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
@@ -508,6 +522,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->unroll = 0;      // auto: 32 with the 40-register kernel, 16 with the 64-register one (measured)
   t->occupancy = 0;   // auto: 40-register kernel when the CSR does not fit in half the L2
   t->root_order = 0;  // auto
+  t->l2_persist_mb = 0;  // auto
   t->root_chunk = 0;  // auto: 1 with the 64-register kernel, 2 with the 40-register one (measured)
   t->block_warps = 16;
   t->blocks_per_sm = 0;
@@ -600,6 +615,28 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   // root order: ascending by default -- descending (high-degree roots first on the
   // ranked copy) measured 1.2-1.7x slower on C2/C3 and neutral on C5
   kp.root_desc = t.root_order == 2 ? 1 : 0;
+  // L2 persistence (B200 126 MB L2): on the degree-ranked copy the rows are in degree
+  // order, so the tail of col_idx holds the longest lists -- the ones every set
+  // operation probes.  Keep up to l2_persist_mb of it persisting in L2 when the CSR
+  // does not fit (auto: off -- measured no gain).
+  {
+    const int64_t csr = (int64_t)g->nnz * 4 + (g->n + 1) * 8;
+    const int mb = t.l2_persist_mb == 0 ? STM_L2_PERSIST_AUTO_MB : t.l2_persist_mb;
+    if (use_rank && mb > 0 && csr > (int64_t)g->l2_bytes / 2 && g->max_window > 0) {
+      int64_t w = std::min<int64_t>((int64_t)mb << 20, std::min<int64_t>(g->max_window, g->nnz * 4));
+      w = std::min<int64_t>(w, g->persist_max);
+      if (w > 0) {
+        if (g->persist_set != w) {
+          if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)w) == cudaSuccess) g->persist_set = w;
+          else cudaGetLastError();
+        }
+        if (g->persist_set > 0) {
+          kp.l2_window_base = (const void*)(g->d_rcol_idx + g->nnz - w / 4);
+          kp.l2_window_bytes = std::min<int64_t>(w, g->persist_set);
+        }
+      }
+    }
+  }
   kp.root_batch = std::max(1, std::min(STM_RMAX, root_chunk));
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
