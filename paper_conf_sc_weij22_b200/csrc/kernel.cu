@@ -56,6 +56,9 @@
 #else
 #define STEP_INL
 #endif
+#ifndef STM_OCC_MAXT
+#define STM_OCC_MAXT 1536   // __launch_bounds__ of the high-occupancy variant (40 registers)
+#endif
 #ifndef STM_ILP2
 #define STM_ILP2 0          // 1: element loop handles two 32-element slices per iteration (probe ILP)
 #endif
@@ -690,6 +693,7 @@ __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
     if (lo >= 0) b = lbound(p, len, lo + 1);
     if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
   }
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->cur[F] = u;
     w.h->it[F] = b;
@@ -750,6 +754,7 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
   const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
   if (nb == ne) return;
   const int u = F >= 1 ? w.h->cur[F] : 0;
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->lgen[F + 1] += 1;  // level F+1 sets are overwritten: drop stale hashes
   __syncwarp();
   for (int st = 0; st < P.n_stages[F + 1]; ++st) {
@@ -845,10 +850,12 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
       const int ub0 = node_ub_const(w, s, F, u);
       if (w.lane < m) NOFF(w, s, w.lane) = w.lane * ub0;
     }
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) w.h->it[F] = pos;
     __syncwarp();
     return m;
   }
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0)
     for (int s = nb; s < ne; ++s) w.h->used[s] = 0;
   __syncwarp();
@@ -915,6 +922,7 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
     }
     __syncwarp();
   }
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->it[F] = pos;
   __syncwarp();
   return m;
@@ -944,6 +952,7 @@ __device__ int gather_roots(W& w) {
     m += __popc(acc);
     pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
   }
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->root_it = pos;
   __syncwarp();
   return m;
@@ -979,6 +988,7 @@ __device__ STEP_INL void fused_count(W& w, int F) {
       int pos = w.h->it[F], e = w.h->end[F];
       if (pos >= e) {
         if (u + 1 >= w.h->nsib[F]) {
+          __syncwarp();  // every lane has read the header fields lane 0 rewrites
           if (w.lane == 0) w.h->cur[F] = u + 1;
           __syncwarp();
           break;
@@ -1012,6 +1022,7 @@ __device__ STEP_INL void fused_count(W& w, int F) {
       }
       nj += __popc(acc);
       int npos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+      __syncwarp();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->it[F] = npos;
       __syncwarp();
       if (nj == 32) break;
@@ -1061,6 +1072,7 @@ __device__ __noinline__ bool try_chunk(W& w) {
 #endif
   if (b < 0) return false;
   lock_ws(w, w.h);
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->root_it = b;
     w.h->root_end = e;
@@ -1163,6 +1175,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   const int k = w.P->k;
   if (T.level == 0) {
     lock_ws(w, w.h);
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->root_it = T.b;
       w.h->root_end = T.e;
@@ -1173,6 +1186,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   }
   const int l = T.level;
   for (int i = 1; i <= l; ++i) {
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       SIB(w, i, 0) = T.prefix[i - 1];
       w.h->nsib[i] = 1;
@@ -1181,12 +1195,14 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
     __syncwarp();
     if (i >= 2) {
       const StmPlan& P = *w.P;
+      __syncwarp();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0)
         for (int s = P.level_begin[i]; s < P.level_begin[i + 1]; ++s) NOFF(w, s, 0) = 0;
       __syncwarp();
       build_nodes(w, i - 1, 1);
     }
     int len = src_len(w, i, 0);
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->it[i] = (i == l) ? T.b : len;
       w.h->end[i] = (i == l) ? min(T.e, len) : len;
@@ -1195,6 +1211,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   }
   (void)k;
   lock_ws(w, w.h);
+  __syncwarp();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->L = l;
   unlock_ws(w, w.h);
 }
@@ -1469,6 +1486,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       int m = gather_roots(w);
       PROF_END(0, m)
       if (m > 0) {
+        __syncwarp();  // every lane has read the header fields lane 0 rewrites
         if (w.lane == 0) {
           w.h->nsib[1] = m;
           w.h->cur[1] = 0;
@@ -1482,6 +1500,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
           frame_count(w, m);  // counts N(root) per root
           continue;
         }
+        __syncwarp();  // every lane has read the header fields lane 0 rewrites
         if (w.lane == 0) w.h->L = 1;
         __syncwarp();
       }
@@ -1505,6 +1524,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       PROF_END(5, 0)
       const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
       if (lk) lock_ws(w, w.h);
+      __syncwarp();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
       if (lk) unlock_ws(w, w.h);
       __syncwarp();
@@ -1529,6 +1549,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       }
       int nu = w.h->cur[F] + 1;
       if (nu >= w.h->nsib[F]) {
+        __syncwarp();  // every lane has read the header fields lane 0 rewrites
         if (w.lane == 0) w.h->cur[F] = nu;
         __syncwarp();
         back = true;
@@ -1539,6 +1560,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       PROF_END(8, 1)
     }
     if (back) {
+      __syncwarp();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
       __syncwarp();
       if (lk) unlock_ws(w, w.h);
@@ -1557,11 +1579,13 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     }
     const bool lk2 = locked_frame(w, F + 1);
     if (lk2) lock_ws(w, w.h);
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) w.h->nsib[F + 1] = m;
     __syncwarp();
     PROF_BEGIN(9)
     set_sibling(w, F + 1, 0);
     PROF_END(9, 1)
+    __syncwarp();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) w.h->L = F + 1;
     __syncwarp();
     if (lk2) unlock_ws(w, w.h);
@@ -1605,7 +1629,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
 __global__ void __launch_bounds__(STM_MAXT, 1) STM_SYM(stm_count_kernel)(const __grid_constant__ StmKParams kp) {
   stm_count_body(kp);
 }
-__global__ void __launch_bounds__(1536, 1) STM_SYM(stm_count_kernel_occ)(const __grid_constant__ StmKParams kp) {
+__global__ void __launch_bounds__(STM_OCC_MAXT, 1) STM_SYM(stm_count_kernel_occ)(const __grid_constant__ StmKParams kp) {
   stm_count_body(kp);
 }
 
