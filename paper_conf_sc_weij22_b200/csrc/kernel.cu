@@ -384,10 +384,19 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   const int* D = An;
   const int* Pp = Bn;
   int dlen = an, plen = bn, use_h = 0;
+  // every job's A ends at the same address: one shared (suffix of a) list, hot in L1
+  const unsigned long long aend = mine ? (unsigned long long)(J.A + J.alen) : 0ull;
+  const unsigned long long aend0 = __shfl_sync(FULLMASK, aend, 0);
+  const bool hotA = w.kp->drive_ratio > 1 && __all_sync(FULLMASK, !mine || aend == aend0);
   int pslot = -1;  // bitmap slot of the probed operand
   if (mine) {
     pslot = J.bbm;
-    if (J.op == STM_OP_AND && bn < an) { D = Bn; dlen = bn; Pp = An; plen = an; pslot = J.abm; }
+    // drive the shorter operand; with a warp-shared (L1-hot) A, drive B while it is at
+    // most drive_ratio times longer: coalesced reads of B and L1-resident probes into A
+    // instead of DRAM-missing probes into B (stm_tuning.drive_ratio)
+    if (J.op == STM_OP_AND && (bn < an || (hotA && bn <= an * w.kp->drive_ratio))) {
+      D = Bn; dlen = bn; Pp = An; plen = an; pslot = J.abm;
+    }
     if (!J.B) { Pp = nullptr; plen = 0; pslot = -1; }
     // a probed hub row is tested in its bitmap: one word per element instead of
     // ceil(log2 |P|) dependent loads (the driving element already lies in (lo, hi))

@@ -76,6 +76,7 @@ struct StmKParams {
   int32_t count_bytes;            // 1 = accumulate algorithmic bytes (instrumented launch)
   int32_t ht_slots;               // per-warp shared-memory hash slots (0 = off)
   int32_t donate_mask;            // donors look for idle blocks every (mask+1)-th opportunity
+  int32_t drive_ratio;            // drive B while |B| <= drive_ratio |A| when A is shared by all jobs (0/1 = shorter)
   int32_t backoff_max;            // idle warps sleep up to 32 << backoff_max ns between steal attempts
   long long watchdog_cycles;      // debug: abort (set work->overflow = 2) after this many cycles; 0 = off
   const void* l2_window_base;     // L2 persisting access-policy window (0 bytes = none)

@@ -523,6 +523,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->occupancy = 0;   // auto: 40-register kernel when the CSR does not fit in half the L2
   t->root_order = 0;  // auto
   t->l2_persist_mb = 0;  // auto
+  t->drive_ratio = 0;    // off (measured)
   t->root_chunk = 0;  // auto: 1 with the 64-register kernel, 2 with the 40-register one (measured)
   t->block_warps = 16;
   t->blocks_per_sm = 0;
@@ -646,13 +647,14 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.ht_slots = t.hash_slots;
   kp.donate_mask = 0;  // look for idle blocks at every opportunity (measured: rate limiting starves idle blocks)
   kp.backoff_max = 8;
+  kp.drive_ratio = t.drive_ratio;
   if (const char* x = getenv("STM_DONATE_MASK")) kp.donate_mask = atoi(x);  // experiments
   if (const char* x = getenv("STM_BACKOFF_MAX")) kp.backoff_max = atoi(x);
   if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
 
   int bps = 0;
   int oe = (la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
-  if (oe != 0) return stm_fail(STM_ECUDA, "occupancy: %s", cudaGetErrorString((cudaError_t)oe));
+  if (oe != 0) return stm_fail(STM_ECUDA, "occupancy (variant %d, %s build, %d warps): %s", variant, la ? "list" : t.instrument ? "instr" : "count", t.block_warps, cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
   const int grid = bps * g->num_sms;

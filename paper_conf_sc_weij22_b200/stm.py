@@ -36,7 +36,7 @@ class stm_tuning(ctypes.Structure):
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
                                                "instrument", "hash_slots", "vertex_order",
                                                "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
-                                               "l2_persist_mb", "narrow_split")]
+                                               "l2_persist_mb", "drive_ratio", "narrow_split")]
 
 
 class stm_shard(ctypes.Structure):

@@ -127,7 +127,7 @@ TUNINGS = [
     dict(occupancy=2), dict(occupancy=2, unroll=32, vertex_order=1), dict(occupancy=1, unroll=32),
     dict(occupancy=2, unroll=5, root_chunk=1, stop_level=3, detect_level=3),
     dict(root_order=1), dict(root_order=2, vertex_order=1), dict(root_order=2, root_chunk=3, occupancy=2),
-    dict(l2_persist_mb=8, occupancy=2),
+    dict(l2_persist_mb=8, occupancy=2), dict(drive_ratio=4), dict(drive_ratio=64, vertex_order=1, occupancy=2),
 ]
 
 

@@ -1,6 +1,3 @@
 mkdir -p gpurun_out
-run() { tool=$1; mode=$2; tag=$3; echo "== $tool $mode $tag"; timeout 900 compute-sanitizer --tool $tool --print-limit 10 python tools/sanitize.py $mode > gpurun_out/sanitize_${tool}_${mode}$tag.log 2>&1; echo "rc=$?"; grep -E "SANITIZE|ERROR SUMMARY|RACECHECK SUMMARY|Error:|list|occupancy" gpurun_out/sanitize_${tool}_${mode}$tag.log | head -8; }
-CUDA_MODULE_LOADING=EAGER run memcheck list _eager
-run racecheck nosteal _v2
-run racecheck count _v2
-python tools/sanitize.py list
+bash tools/gpu_var2.sh d1 c5:k5,c5:k6_minus_e,c3:k5,c2:c4 "cur" "cur|drive_ratio=2" "cur|drive_ratio=4" "cur|drive_ratio=8" "occ64" "occ56|block_warps=14" "occ64|drive_ratio=4"
+timeout 900 compute-sanitizer --tool memcheck --print-limit 10 python tools/sanitize.py list > gpurun_out/sanitize_memcheck_list.log 2>&1; echo "memcheck list rc=$?"; grep -E "SANITIZE|ERROR SUMMARY|list" gpurun_out/sanitize_memcheck_list.log | head

@@ -20,7 +20,8 @@ for name, vi in [("k4", False), ("house", True), ("c5", False)]:
         print(name, vi, tk, got, want, flush=True)
         ok &= got == want
     if mode == "list":
-        rows, c = stm.stm_match_list(G.handle, stm.Plan(p.k, p.edges, vertex_induced=vi).handle, p.k, None, capacity=50)
+        plan = stm.Plan(p.k, p.edges, vertex_induced=vi)  # keep the handle's owner alive
+        rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, None, capacity=50)
         print(name, vi, "list", c, want, flush=True)
         ok &= c == want
 print("SANITIZE_COUNTS_OK" if ok else "SANITIZE_COUNTS_MISMATCH")
