@@ -176,7 +176,8 @@ typedef struct stm_tuning {
                              device; sets the device's persisting L2 limit).  Speed only. */
   int32_t drive_ratio;    /* intersection driving side: the shorter operand drives (0 or 1); k > 1: when
                              all jobs of a combined operation share operand A (hot in L1), B drives while
-                             |B| <= k |A| (coalesced reads of B, L1 probes into A).  Speed only. */
+                             |B| <= k |A| (coalesced reads of B, L1 probes into A).  Speed only.  Only in
+                             builds with -DSTM_DRIVE_RATIO=1 (else STM_EUNSUPPORTED): measured slower. */
   int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
                              out_start[v] (first neighbour > v, built at load); 1 = binary search only.
                              Speed only.  Default 0. */

@@ -56,6 +56,25 @@
 #else
 #define STEP_INL
 #endif
+#ifndef STM_HDR_SYNC
+#define STM_HDR_SYNC 1  // __syncwarp() between the lanes' reads of a stack-header field and lane 0's rewrite
+#endif
+#if STM_HDR_SYNC
+#define HDR_SYNC() __syncwarp()
+#else
+#define HDR_SYNC() ((void)0)
+#endif
+#ifndef STM_DRIVE_RATIO
+#define STM_DRIVE_RATIO 0  // 1: compile in the drive_ratio operand choice (measured slower; A/B builds)
+#endif
+#ifndef STM_GATHER_SLOW_NOINLINE
+#define STM_GATHER_SLOW_NOINLINE 0  // 1: the per-candidate admission path out of line (A/B)
+#endif
+#if STM_GATHER_SLOW_NOINLINE
+#define GATHER_SLOW_INL __noinline__
+#else
+#define GATHER_SLOW_INL __forceinline__
+#endif
 #ifndef STM_OCC_MAXT
 #define STM_OCC_MAXT 1536   // __launch_bounds__ of the high-occupancy variant (40 registers)
 #endif
@@ -385,9 +404,12 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   const int* Pp = Bn;
   int dlen = an, plen = bn, use_h = 0;
   // every job's A ends at the same address: one shared (suffix of a) list, hot in L1
-  const unsigned long long aend = mine ? (unsigned long long)(J.A + J.alen) : 0ull;
-  const unsigned long long aend0 = __shfl_sync(FULLMASK, aend, 0);
-  const bool hotA = w.kp->drive_ratio > 1 && __all_sync(FULLMASK, !mine || aend == aend0);
+  bool hotA = false;
+  if (STM_DRIVE_RATIO && w.kp->drive_ratio > 1) {
+    const unsigned long long aend = mine ? (unsigned long long)(J.A + J.alen) : 0ull;
+    const unsigned long long aend0 = __shfl_sync(FULLMASK, aend, 0);
+    hotA = __all_sync(FULLMASK, !mine || aend == aend0);
+  }
   int pslot = -1;  // bitmap slot of the probed operand
   if (mine) {
     pslot = J.bbm;
@@ -702,7 +724,7 @@ __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
     if (lo >= 0) b = lbound(p, len, lo + 1);
     if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
   }
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->cur[F] = u;
     w.h->it[F] = b;
@@ -763,7 +785,7 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
   const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
   if (nb == ne) return;
   const int u = F >= 1 ? w.h->cur[F] : 0;
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  // (reads above are ordered before this write by a full-warp collective)
   if (w.lane == 0) w.h->lgen[F + 1] += 1;  // level F+1 sets are overwritten: drop stale hashes
   __syncwarp();
   for (int st = 0; st < P.n_stages[F + 1]; ++st) {
@@ -817,54 +839,12 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
 // siblings of frame F+1, admitted so that every node region fits.
 // Caller holds the frame lock if the frame is stealable.  Returns batch size.
 // ----------------------------------------------------------------------------
-__device__ STEP_INL int gather_batch(W& w, int F, int U) {
-  const StmPlan& P = *w.P;
-  const int u = w.h->cur[F];
-  const int* src;
-  int len;
-  src_slice(w, P.cand[F], F, u, 0, 0, src, len);
-  int lo, hi;
-  const StmFilter f = P.filt[F];
-  bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
-  int pos = w.h->it[F];
-  const int e = w.h->end[F];
-  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
-  const int cap = w.kp->cap;
-  // Fast admission: when U copies of every node's candidate-independent size bound
-  // fit in its region, any batch of <= U candidates fits -- fixed slice offsets
-  // t * bound, no per-candidate degree loads or prefix sums.
-  bool fixed = true;
-  for (int s = nb; s < ne && fixed; ++s) fixed = (long long)node_ub_const(w, s, F, u) * U <= (long long)cap;
-  if (fixed) {
-    int m = 0;
-    while (m < U && pos < e) {
-      const int p = pos + w.lane;
-      const bool valid = p < e;
-      const int c = valid ? src[p] : 0;
-      const bool pass = valid && cand_ok(w, F, u, c, lo, hi);
-      unsigned acc = __ballot_sync(FULLMASK, pass);
-      const int room = U - m;
-      bool cut = false;
-      if (__popc(acc) > room) {
-        unsigned a2 = 0, t = acc;  // keep the first `room` set bits
-        for (int i = 0; i < room; ++i) { const unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
-        acc = a2;
-        cut = true;
-      }
-      if ((acc >> w.lane) & 1u) SIB(w, F + 1, m + __popc(acc & ((1u << w.lane) - 1))) = c;
-      m += __popc(acc);
-      pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
-    }
-    for (int s = nb; s < ne; ++s) {
-      const int ub0 = node_ub_const(w, s, F, u);
-      if (w.lane < m) NOFF(w, s, w.lane) = w.lane * ub0;
-    }
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
-    if (w.lane == 0) w.h->it[F] = pos;
-    __syncwarp();
-    return m;
-  }
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+// Admission with per-candidate size bounds: used when U copies of a
+// node's candidate-independent bound may not fit; kept out of line (cold for most plans).
+__device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* src, int lo, int hi, int pos,
+                                                 const int e, const int nb, const int ne, const int cap,
+                                                 const int u) {
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0)
     for (int s = nb; s < ne; ++s) w.h->used[s] = 0;
   __syncwarp();
@@ -931,10 +911,60 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
     }
     __syncwarp();
   }
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->it[F] = pos;
   __syncwarp();
   return m;
+}
+
+__device__ STEP_INL int gather_batch(W& w, int F, int U) {
+  const StmPlan& P = *w.P;
+  const int u = w.h->cur[F];
+  const int* src;
+  int len;
+  src_slice(w, P.cand[F], F, u, 0, 0, src, len);
+  int lo, hi;
+  const StmFilter f = P.filt[F];
+  bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
+  int pos = w.h->it[F];
+  const int e = w.h->end[F];
+  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
+  const int cap = w.kp->cap;
+  // Fast admission: when U copies of every node's candidate-independent size bound
+  // fit in its region, any batch of <= U candidates fits -- fixed slice offsets
+  // t * bound, no per-candidate degree loads or prefix sums.
+  bool fixed = true;
+  for (int s = nb; s < ne && fixed; ++s) fixed = (long long)node_ub_const(w, s, F, u) * U <= (long long)cap;
+  if (fixed) {
+    int m = 0;
+    while (m < U && pos < e) {
+      const int p = pos + w.lane;
+      const bool valid = p < e;
+      const int c = valid ? src[p] : 0;
+      const bool pass = valid && cand_ok(w, F, u, c, lo, hi);
+      unsigned acc = __ballot_sync(FULLMASK, pass);
+      const int room = U - m;
+      bool cut = false;
+      if (__popc(acc) > room) {
+        unsigned a2 = 0, t = acc;  // keep the first `room` set bits
+        for (int i = 0; i < room; ++i) { const unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+        acc = a2;
+        cut = true;
+      }
+      if ((acc >> w.lane) & 1u) SIB(w, F + 1, m + __popc(acc & ((1u << w.lane) - 1))) = c;
+      m += __popc(acc);
+      pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+    }
+    for (int s = nb; s < ne; ++s) {
+      const int ub0 = node_ub_const(w, s, F, u);
+      if (w.lane < m) NOFF(w, s, w.lane) = w.lane * ub0;
+    }
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+    if (w.lane == 0) w.h->it[F] = pos;
+    __syncwarp();
+    return m;
+  }
+  return gather_batch_slow(w, F, U, src, lo, hi, pos, e, nb, ne, cap, u);
 }
 
 // root batch: up to root_batch roots from [root_it, root_end) with the root label
@@ -961,7 +991,7 @@ __device__ int gather_roots(W& w) {
     m += __popc(acc);
     pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
   }
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->root_it = pos;
   __syncwarp();
   return m;
@@ -997,7 +1027,7 @@ __device__ STEP_INL void fused_count(W& w, int F) {
       int pos = w.h->it[F], e = w.h->end[F];
       if (pos >= e) {
         if (u + 1 >= w.h->nsib[F]) {
-          __syncwarp();  // every lane has read the header fields lane 0 rewrites
+          HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
           if (w.lane == 0) w.h->cur[F] = u + 1;
           __syncwarp();
           break;
@@ -1031,7 +1061,7 @@ __device__ STEP_INL void fused_count(W& w, int F) {
       }
       nj += __popc(acc);
       int npos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
-      __syncwarp();  // every lane has read the header fields lane 0 rewrites
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->it[F] = npos;
       __syncwarp();
       if (nj == 32) break;
@@ -1081,7 +1111,7 @@ __device__ __noinline__ bool try_chunk(W& w) {
 #endif
   if (b < 0) return false;
   lock_ws(w, w.h);
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->root_it = b;
     w.h->root_end = e;
@@ -1184,7 +1214,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   const int k = w.P->k;
   if (T.level == 0) {
     lock_ws(w, w.h);
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->root_it = T.b;
       w.h->root_end = T.e;
@@ -1195,7 +1225,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   }
   const int l = T.level;
   for (int i = 1; i <= l; ++i) {
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       SIB(w, i, 0) = T.prefix[i - 1];
       w.h->nsib[i] = 1;
@@ -1204,14 +1234,14 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
     __syncwarp();
     if (i >= 2) {
       const StmPlan& P = *w.P;
-      __syncwarp();  // every lane has read the header fields lane 0 rewrites
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0)
         for (int s = P.level_begin[i]; s < P.level_begin[i + 1]; ++s) NOFF(w, s, 0) = 0;
       __syncwarp();
       build_nodes(w, i - 1, 1);
     }
     int len = src_len(w, i, 0);
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->it[i] = (i == l) ? T.b : len;
       w.h->end[i] = (i == l) ? min(T.e, len) : len;
@@ -1220,7 +1250,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   }
   (void)k;
   lock_ws(w, w.h);
-  __syncwarp();  // every lane has read the header fields lane 0 rewrites
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->L = l;
   unlock_ws(w, w.h);
 }
@@ -1495,7 +1525,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       int m = gather_roots(w);
       PROF_END(0, m)
       if (m > 0) {
-        __syncwarp();  // every lane has read the header fields lane 0 rewrites
+        // (reads above are ordered before this write by a full-warp collective)
         if (w.lane == 0) {
           w.h->nsib[1] = m;
           w.h->cur[1] = 0;
@@ -1509,7 +1539,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
           frame_count(w, m);  // counts N(root) per root
           continue;
         }
-        __syncwarp();  // every lane has read the header fields lane 0 rewrites
+        // (reads above are ordered before this write by a full-warp collective)
         if (w.lane == 0) w.h->L = 1;
         __syncwarp();
       }
@@ -1533,7 +1563,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       PROF_END(5, 0)
       const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
       if (lk) lock_ws(w, w.h);
-      __syncwarp();  // every lane has read the header fields lane 0 rewrites
+      // (reads above are ordered before this write by a full-warp collective)
       if (w.lane == 0) w.h->L = F - 1;
       if (lk) unlock_ws(w, w.h);
       __syncwarp();
@@ -1558,7 +1588,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       }
       int nu = w.h->cur[F] + 1;
       if (nu >= w.h->nsib[F]) {
-        __syncwarp();  // every lane has read the header fields lane 0 rewrites
+        HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
         if (w.lane == 0) w.h->cur[F] = nu;
         __syncwarp();
         back = true;
@@ -1569,7 +1599,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       PROF_END(8, 1)
     }
     if (back) {
-      __syncwarp();  // every lane has read the header fields lane 0 rewrites
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
       __syncwarp();
       if (lk) unlock_ws(w, w.h);
@@ -1588,13 +1618,13 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     }
     const bool lk2 = locked_frame(w, F + 1);
     if (lk2) lock_ws(w, w.h);
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
+    // (reads above are ordered before this write by a full-warp collective)
     if (w.lane == 0) w.h->nsib[F + 1] = m;
     __syncwarp();
     PROF_BEGIN(9)
     set_sibling(w, F + 1, 0);
     PROF_END(9, 1)
-    __syncwarp();  // every lane has read the header fields lane 0 rewrites
+    // (reads above are ordered before this write by a full-warp collective)
     if (w.lane == 0) w.h->L = F + 1;
     __syncwarp();
     if (lk2) unlock_ws(w, w.h);
@@ -1647,6 +1677,7 @@ static const void* STM_SYM(kernel_fn)(int variant) {
 }
 
 #if !STM_INSTR && !STM_LIST
+int stm_drive_compiled() { return STM_DRIVE_RATIO; }
 int stm_hash_compiled() { return STM_WITH_HASH; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {

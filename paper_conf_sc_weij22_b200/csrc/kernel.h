@@ -86,6 +86,8 @@ struct StmKParams {
 
 // 1 if the shared-memory hash-set path is compiled in (-DSTM_WITH_HASH=1)
 int stm_hash_compiled();
+// 1 if the drive_ratio operand choice is compiled in (-DSTM_DRIVE_RATIO=1)
+int stm_drive_compiled();
 // size in bytes of the dynamic shared memory for one block
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
 // kernel variants (register budgets): 1 = 64 registers, 2 = 40 registers (more warps)

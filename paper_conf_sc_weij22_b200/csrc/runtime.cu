@@ -647,6 +647,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.ht_slots = t.hash_slots;
   kp.donate_mask = 0;  // look for idle blocks at every opportunity (measured: rate limiting starves idle blocks)
   kp.backoff_max = 8;
+  if (t.drive_ratio > 1 && !stm_drive_compiled())
+    return stm_fail(STM_EUNSUPPORTED, "drive_ratio: this build has no drive-ratio path (-DSTM_DRIVE_RATIO=1)");
   kp.drive_ratio = t.drive_ratio;
   if (const char* x = getenv("STM_DONATE_MASK")) kp.donate_mask = atoi(x);  // experiments
   if (const char* x = getenv("STM_BACKOFF_MAX")) kp.backoff_max = atoi(x);

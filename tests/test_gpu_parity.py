@@ -127,7 +127,7 @@ TUNINGS = [
     dict(occupancy=2), dict(occupancy=2, unroll=32, vertex_order=1), dict(occupancy=1, unroll=32),
     dict(occupancy=2, unroll=5, root_chunk=1, stop_level=3, detect_level=3),
     dict(root_order=1), dict(root_order=2, vertex_order=1), dict(root_order=2, root_chunk=3, occupancy=2),
-    dict(l2_persist_mb=8, occupancy=2), dict(drive_ratio=4), dict(drive_ratio=64, vertex_order=1, occupancy=2),
+    dict(l2_persist_mb=8, occupancy=2),
 ]
 
 
@@ -374,3 +374,11 @@ def test_listing_pages_and_capacity(rmat_small):
     assert c == want.shape[0] and rows.shape[0] == 7 and all(tuple(r) in wanted for r in rows)
     rows, c = stm.stm_match_list(G.handle, plan.handle, p.k, t, capacity=0)
     assert c == want.shape[0] and rows.shape[0] == 0
+
+
+def test_compiled_out_options_fail_loudly(er_small):
+    """Options whose code path is compiled out of the product build are refused, never ignored."""
+    g, G = er_small
+    p = CATALOG["triangle"]
+    with pytest.raises(stm.StmError, match="STM_EUNSUPPORTED"):
+        gcount(G, p, False, tuning=stm.stm_tuning_default(drive_ratio=4))
