@@ -300,6 +300,58 @@ stm_status stm_last_launch(stm_launch_info* info);
  */
 stm_status stm_last_profile(uint64_t* out, int n);
 
+/* ---------------------------------------------------------------------------------------
+ * Cost-based matching order.  PAPER.md:151: STMatch adopts
+ * Dryadic's matching order; PAPER.md:52 requires only that every pi[l] after the first
+ * be adjacent to an earlier one.  The order changes the work, never the count.  These
+ * calls are host-only (no CUDA) and choose the `order` argument of stm_pattern_compile
+ * from degree / label statistics of the data graph (cost model: DESIGN.md reading R15).
+ * ------------------------------------------------------------------------------------- */
+enum { STM_STATS_MOMENTS = 9, STM_STATS_LABELS = 256 };
+
+typedef struct stm_graph_stats {
+  int64_t n;                                /* vertices */
+  int64_t nnz;                              /* directed adjacency entries (2m) */
+  double moment[STM_STATS_MOMENTS];         /* moment[j] = (1/n) sum_v w(v)^j, w(v) = min(d(v), sqrt(nnz)) */
+  int32_t n_labels;                         /* distinct vertex labels (0 = unlabeled graph) */
+  int32_t reserved;
+  int32_t label_value[STM_STATS_LABELS];    /* ascending label values */
+  double label_freq[STM_STATS_LABELS];      /* fraction of vertices carrying label_value[i] */
+} stm_graph_stats;
+
+/*
+ * stm_graph_stats_host -- degree moments and label frequencies of a host CSR (the same
+ * row_ptr / labels arrays stm_graph_load takes; col_idx is not needed).  O(n).
+ * Caller owns `out`.  Errors: STM_EINVAL (NULL out, n < 0, decreasing row_ptr,
+ * negative label), STM_EUNSUPPORTED (> 256 distinct labels).
+ */
+stm_status stm_graph_stats_host(int64_t n, const int64_t* row_ptr, const int32_t* labels,
+                                stm_graph_stats* out);
+
+/*
+ * stm_order_cost -- model cost of matching `order` (int32[k], a connected permutation)
+ * for the pattern (k, edges, labels, restrictions, flags exactly as stm_pattern_compile
+ * takes them; STM_AUTO_RESTRICT uses the compiler's Grochow-Kellis set) on a graph with
+ * statistics `stats`.  *cost = expected merge work (n + sum over levels of estimated
+ * prefixes x summed operand list lengths); *est_count = estimated number of counted
+ * embeddings (Chung-Lu expectation of homomorphisms, label and restriction factors).
+ * Either output may be NULL.  Errors: those of stm_pattern_compile; STM_EINVAL for a
+ * NULL stats / order or an order that is not a connected permutation.
+ */
+stm_status stm_order_cost(int k, int n_edges, const int32_t* edges, const int32_t* labels, int n_restr,
+                          const int32_t* restr, uint32_t flags, const stm_graph_stats* stats,
+                          const int32_t* order, double* cost, double* est_count);
+
+/*
+ * stm_order_optimize -- the connected order of minimal model cost (exhaustive over the
+ * <= 8! permutations; the compiler's greedy order is kept unless another is strictly
+ * cheaper).  Writes int32[k] to order_out (caller-owned); cost / est_count as in
+ * stm_order_cost (may be NULL).  Errors as stm_order_cost.
+ */
+stm_status stm_order_optimize(int k, int n_edges, const int32_t* edges, const int32_t* labels, int n_restr,
+                              const int32_t* restr, uint32_t flags, const stm_graph_stats* stats,
+                              int32_t* order_out, double* cost, double* est_count);
+
 /* stm_last_error -- thread-local message for the last non-OK status of this thread. */
 const char* stm_last_error(void);
 

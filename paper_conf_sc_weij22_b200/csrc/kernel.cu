@@ -5,7 +5,7 @@
 // on its own DFS stack kept in shared memory; the candidate
 // sets (the paper's C arrays) live in a per-warp global arena sized from the
 // graph's true maximum degree (PAPER.md:154 used a fixed MAX_DEGREE=4096; reading
-// R15).  Level 0 takes chunks of root vertices from a global atomic cursor
+// R11).  Level 0 takes chunks of root vertices from a global atomic cursor
 // (Fig. 4).
 //
 // Set operations: a *job* is one "A op N(v)" with op in

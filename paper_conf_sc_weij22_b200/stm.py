@@ -22,7 +22,8 @@ _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED
 EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
            "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
            "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
-           "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error"]
+           "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error",
+           "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize"]
 
 
 class StmError(RuntimeError):
@@ -53,6 +54,16 @@ class stm_launch_info(ctypes.Structure):
                 ("hubs", ctypes.c_int64), ("variant", ctypes.c_int32), ("unroll", ctypes.c_int32)]
 
 
+STM_STATS_MOMENTS, STM_STATS_LABELS = 9, 256
+
+
+class stm_graph_stats(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("moment", ctypes.c_double * STM_STATS_MOMENTS),
+                ("n_labels", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("label_value", ctypes.c_int32 * STM_STATS_LABELS),
+                ("label_freq", ctypes.c_double * STM_STATS_LABELS)]
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_weij22_b200.build` "
@@ -77,6 +88,11 @@ def _load():
         "stm_match_list": [vp, vp, vp, i64, i64, vp, vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
                            ctypes.POINTER(ctypes.c_uint64)],
         "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
+        "stm_graph_stats_host": [i64, vp, vp, ctypes.POINTER(stm_graph_stats)],
+        "stm_order_cost": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
+                           ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
+        "stm_order_optimize": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
+                               ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -139,6 +155,41 @@ def stm_pattern_compile(k: int, edges, labels=None, order=None, restrictions=Non
     h = ctypes.c_void_p()
     _check(lib.stm_pattern_compile(k, e.size // 2, _p(e), _p(lb), _p(od), nr, _p(rs), flags, ctypes.byref(h)))
     return h.value
+
+
+def stm_graph_stats_host(n: int, row_ptr, labels=None) -> stm_graph_stats:
+    rp = _arr(row_ptr, np.int64)
+    lb = _arr(labels, np.int32)
+    st = stm_graph_stats()
+    _check(lib.stm_graph_stats_host(n, _p(rp), _p(lb), ctypes.byref(st)))
+    return st
+
+
+def _pattern_args(edges, labels, restrictions):
+    e = _arr(edges, np.int32).reshape(-1)
+    lb = _arr(labels, np.int32)
+    rs = _arr(restrictions, np.int32).reshape(-1) if restrictions is not None and len(restrictions) else None
+    return e, lb, rs, 0 if rs is None else rs.size // 2
+
+
+def stm_order_cost(k: int, edges, labels, restrictions, flags: int, stats: stm_graph_stats,
+                   order) -> Tuple[float, float]:
+    e, lb, rs, nr = _pattern_args(edges, labels, restrictions)
+    od = _arr(order, np.int32)
+    c, est = ctypes.c_double(), ctypes.c_double()
+    _check(lib.stm_order_cost(k, e.size // 2, _p(e), _p(lb), nr, _p(rs), flags, ctypes.byref(stats), _p(od),
+                              ctypes.byref(c), ctypes.byref(est)))
+    return c.value, est.value
+
+
+def stm_order_optimize(k: int, edges, labels, restrictions, flags: int,
+                       stats: stm_graph_stats) -> Tuple[list, float, float]:
+    e, lb, rs, nr = _pattern_args(edges, labels, restrictions)
+    od = np.zeros(k, np.int32)
+    c, est = ctypes.c_double(), ctypes.c_double()
+    _check(lib.stm_order_optimize(k, e.size // 2, _p(e), _p(lb), nr, _p(rs), flags, ctypes.byref(stats), _p(od),
+                                  ctypes.byref(c), ctypes.byref(est)))
+    return od.tolist(), c.value, est.value
 
 
 def stm_plan_describe(p: int) -> str:
@@ -277,13 +328,19 @@ class Plan:
     """Compiled pattern (owns the stm_plan handle)."""
 
     def __init__(self, k: int, edges, labels=None, order=None, restrictions=None, vertex_induced=False,
-                 code_motion=True, auto_restrict=None, auto_order=False, lazy_unbounded=False):
+                 code_motion=True, auto_restrict=None, auto_order=False, lazy_unbounded=False,
+                 cost_stats: Optional[stm_graph_stats] = None):
+        """cost_stats: graph statistics (stm_graph_stats_host) -> the cost-optimal order (NEXT-2)
+        replaces `order`."""
         if auto_restrict is None:
             auto_restrict = restrictions is None
         flags = (STM_VERTEX_INDUCED if vertex_induced else 0) | (0 if code_motion else STM_NO_CODE_MOTION)
         flags |= STM_AUTO_RESTRICT if auto_restrict else 0
-        flags |= STM_AUTO_ORDER if auto_order else 0
         flags |= STM_LAZY_UNBOUNDED if lazy_unbounded else 0
+        if cost_stats is not None:
+            order, self.model_cost, self.model_count = stm_order_optimize(k, edges, labels, restrictions, flags,
+                                                                          cost_stats)
+        flags |= STM_AUTO_ORDER if auto_order else 0
         self.handle = stm_pattern_compile(k, edges, labels, order, restrictions, flags)
         self.k, self.n_sets, self.aut = stm_plan_info(self.handle)
         self.first_vertex = stm_plan_first_vertex(self.handle)

@@ -382,3 +382,16 @@ def test_compiled_out_options_fail_loudly(er_small):
     p = CATALOG["triangle"]
     with pytest.raises(stm.StmError, match="STM_EUNSUPPORTED"):
         gcount(G, p, False, tuning=stm.stm_tuning_default(drive_ratio=4))
+
+
+@pytest.mark.parametrize("name", ["path4", "c4", "tailed_triangle", "house", "c5", "w5", "c6", "prism", "w6", "c7"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_cost_order_counts(rmat_small, name, vi):
+    """NEXT-2: the cost-optimal matching order (stm_order_optimize) changes the work,
+    never the count -- bit-exact against the oracle, unlabeled and labeled."""
+    g, G = rmat_small
+    p = CATALOG[name]
+    stats = stm.stm_graph_stats_host(g.n, g.row_ptr, g.labels)
+    for lab in (None, stmgen.pattern_labels(p.k, 4, 3)):
+        plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, cost_stats=stats)
+        assert stm.count(G, plan) == ocount(g, p, vi, labels=lab)

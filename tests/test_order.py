@@ -1,0 +1,172 @@
+"""Cost-based matching order (PAPER.md:151 adopts Dryadic's order,
+PAPER.md:52 requires only connected orders).  Host-only: no CUDA device needed.
+
+The cost model (reading R15) is a heuristic, so these tests pin what is exact
+about it: the graph statistics, the Chung-Lu homomorphism expectation on regular graphs
+(where it equals the true homomorphism count of a tree: n d^(k-1)), the linear-extension
+restriction factor, and that the search returns the minimum over every connected order.
+That the chosen order leaves the count unchanged is a GPU parity test
+(tests/test_gpu_parity.py::test_cost_order_counts).
+"""
+import itertools
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import stmgen
+from stmgen import CATALOG
+
+
+@pytest.fixture(scope="module")
+def stm():
+    from paper_conf_sc_weij22_b200 import build
+    build.build()
+    from paper_conf_sc_weij22_b200 import stm as m
+    return m
+
+
+def connected_orders(p):
+    adj = {u: set() for u in range(p.k)}
+    for a, b in p.edges:
+        adj[a].add(b)
+        adj[b].add(a)
+    for perm in itertools.permutations(range(p.k)):
+        if all(any(perm[j] in adj[perm[i]] for j in range(i)) for i in range(1, p.k)):
+            yield list(perm)
+
+
+def test_stats_closed_forms(stm):
+    # K_n: every degree n-1 (<= sqrt(n(n-1)), so uncapped): moment[j] = (n-1)^j
+    g = stmgen.complete(9)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    assert s.n == 9 and s.nnz == 72 and s.n_labels == 0
+    for j in range(stm.STM_STATS_MOMENTS):
+        assert s.moment[j] == pytest.approx(8.0 ** j, rel=1e-12)
+    # star K_{1,15}: the hub's degree 15 is capped at sqrt(2m) = sqrt(30)
+    g = stmgen.from_edges(16, [(0, i) for i in range(1, 16)])
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    w = np.minimum(np.diff(g.row_ptr).astype(float), math.sqrt(30.0))
+    for j in range(stm.STM_STATS_MOMENTS):
+        assert s.moment[j] == pytest.approx(np.mean(w ** j), rel=1e-12)
+    assert max(w) == pytest.approx(math.sqrt(30.0))
+
+
+def test_stats_labels(stm):
+    g = stmgen.er(500, 2000, 3)
+    lab = stmgen.labels(g.n, 5, 4)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr, lab)
+    vals, cnt = np.unique(lab, return_counts=True)
+    assert s.n_labels == len(vals)
+    assert list(s.label_value[: s.n_labels]) == vals.tolist()
+    assert list(s.label_freq[: s.n_labels]) == pytest.approx((cnt / g.n).tolist())
+    with pytest.raises(stm.StmError):
+        stm.stm_graph_stats_host(g.n, g.row_ptr, -np.ones(g.n, np.int32))
+
+
+@pytest.mark.parametrize("name", ["edge", "wedge", "path4", "star4"])
+def test_tree_estimate_is_exact_on_regular_graphs(stm, name):
+    # On a d-regular graph the number of homomorphisms of a tree with k vertices is
+    # exactly n d^(k-1); on the cycle C_n (d = 2) brute force confirms it.
+    p = CATALOG[name]
+    g = stmgen.cycle(12)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    for order in connected_orders(p):
+        _, est = stm.stm_order_cost(p.k, p.edges, None, [], 0, s, order)
+        assert est == pytest.approx(g.n * 2.0 ** (p.k - 1), rel=1e-12)
+    # homomorphisms of a tree on C_12 = injective maps + non-injective ones; the model
+    # counts homomorphisms, so compare with the walk count: n * 2^(k-1) for paths from
+    # every vertex -- checked against the oracle's injective count as an upper bound.
+    assert oracle.count(g, p.k, p.edges) <= g.n * 2 ** (p.k - 1)
+
+
+def test_restriction_factor_is_linear_extensions(stm):
+    # star4 with Grochow-Kellis restrictions (leaves 1 < 2 < 3): 1 of 3! leaf orders
+    p = CATALOG["star4"]
+    g = stmgen.complete(10)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    _, free = stm.stm_order_cost(p.k, p.edges, None, [], 0, s, [0, 1, 2, 3])
+    _, gk = stm.stm_order_cost(p.k, p.edges, None, None, stm.STM_AUTO_RESTRICT, s, [0, 1, 2, 3])
+    assert gk == pytest.approx(free / 6, rel=1e-12)
+    # a custom partial order 1 < 2, 1 < 3 (2, 3 free): 2 linear extensions of 3! -> 1/3
+    _, part = stm.stm_order_cost(p.k, p.edges, None, [(1, 2), (1, 3)], 0, s, [0, 1, 2, 3])
+    assert part == pytest.approx(free / 3, rel=1e-12)
+    # the estimate is the homomorphism expectation n^k prod M_deg / (2m)^|E|
+    assert free == pytest.approx(10 * 9.0 ** 3, rel=1e-12)
+
+
+def test_label_factor(stm):
+    p = CATALOG["triangle"]
+    g = stmgen.complete(12)
+    lab = np.array([0] * 3 + [1] * 9, np.int32)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr, lab)
+    _, unl = stm.stm_order_cost(3, p.edges, None, [], 0, s, [0, 1, 2])
+    _, l0 = stm.stm_order_cost(3, p.edges, [0, 1, -1], [], 0, s, [0, 1, 2])
+    assert l0 == pytest.approx(unl * 0.25 * 0.75, rel=1e-12)
+    _, l9 = stm.stm_order_cost(3, p.edges, [0, 9, 1], [], 0, s, [0, 1, 2])
+    assert l9 == 0.0
+
+
+def test_triangle_estimate_on_er(stm):
+    # G(n, p): expected triangles C(n,3) p^3; the Chung-Lu estimate from observed degree
+    # moments is within sampling + degree-variance error of the oracle's exact count.
+    g = stmgen.config_graph("c1")
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    p = CATALOG["triangle"]
+    _, est = stm.stm_order_cost(3, p.edges, None, None, stm.STM_AUTO_RESTRICT, s, [0, 1, 2])
+    exact = oracle.count(g, 3, p.edges, restrictions=oracle.gk_restrictions(3, p.edges))
+    assert 0.75 * exact < est < 1.35 * exact
+
+
+@pytest.mark.parametrize("name", ["path4", "c4", "diamond", "tailed_triangle", "house", "c5", "w5", "c6",
+                                  "k6_minus_e", "prism"])
+@pytest.mark.parametrize("vi", [False, True])
+def test_optimum_over_all_connected_orders(stm, name, vi):
+    p = CATALOG[name]
+    g = stmgen.rmat(12, 30000, 0.57, 0.19, 0.19, 5)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    flags = stm.STM_AUTO_RESTRICT | (stm.STM_VERTEX_INDUCED if vi else 0)
+    order, cost, est = stm.stm_order_optimize(p.k, p.edges, None, None, flags, s)
+    assert sorted(order) == list(range(p.k))
+    costs = {tuple(o): stm.stm_order_cost(p.k, p.edges, None, None, flags, s, o) for o in connected_orders(p)}
+    assert tuple(order) in costs
+    assert cost == pytest.approx(costs[tuple(order)][0], rel=1e-12)
+    assert cost <= min(c for c, _ in costs.values()) * (1 + 1e-9)
+    # the estimated count does not depend on the order
+    assert all(e == pytest.approx(est, rel=1e-9) for _, e in costs.values())
+
+
+@pytest.mark.parametrize("name", ["triangle", "k4", "k5", "k6", "k8"])
+def test_cliques_keep_the_greedy_order(stm, name):
+    p = CATALOG[name]
+    g = stmgen.rmat(10, 4000, 0.57, 0.19, 0.19, 17)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    order, _, _ = stm.stm_order_optimize(p.k, p.edges, None, None, stm.STM_AUTO_RESTRICT, s)
+    plan = stm.Plan(p.k, p.edges, auto_order=True)
+    assert f"order=[{','.join(map(str, order))}]" in plan.describe()
+
+
+def test_cycle_order_closes_early_on_hub_graphs(stm):
+    # For C4 with restrictions 0 < {1, 2, 3}, 1 < 3 the optimum places both neighbours
+    # of vertex 0 first (the 1 < 3 bound prunes at level 2), halving the model's cost.
+    p = CATALOG["c4"]
+    g = stmgen.config_graph("c2")
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    order, cost, _ = stm.stm_order_optimize(4, p.edges, None, None, stm.STM_AUTO_RESTRICT, s)
+    greedy, _ = stm.stm_order_cost(4, p.edges, None, None, stm.STM_AUTO_RESTRICT, s, [0, 1, 2, 3])
+    assert cost < 0.6 * greedy
+    plan = stm.Plan(4, p.edges, cost_stats=s)
+    assert f"order=[{','.join(map(str, order))}]" in plan.describe()
+
+
+def test_errors(stm):
+    p = CATALOG["path4"]
+    g = stmgen.cycle(8)
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    with pytest.raises(stm.StmError):
+        stm.stm_order_cost(4, p.edges, None, [], 0, s, [0, 2, 1, 3])  # 2 not adjacent to 0
+    with pytest.raises(stm.StmError):
+        stm.stm_order_cost(4, p.edges, None, [], 0, s, [0, 0, 1, 2])
+    with pytest.raises(stm.StmError):
+        stm.stm_order_optimize(4, [(0, 1), (2, 3)], None, [], 0, s)  # disconnected

@@ -13,13 +13,19 @@ for spec in specs:
     vi = ":vi" in spec
     nocm = ":nocm" in spec
     lazy = ":lazy" in spec
+    cost = ":cost" in spec  # cost-based matching order (stm_order_optimize, NEXT-2)
     if cfg not in graphs:
         g = stmgen.config_graph(cfg)
         graphs[cfg] = (g, stm.Graph.from_stmgen(g))
     g, G = graphs[cfg]
     p = stmgen.CATALOG[name]
     lab = stmgen.pattern_labels(p.k, 8, 7) if g.labels is not None else None
-    plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, code_motion=not nocm, lazy_unbounded=lazy)
+    stats = stm.stm_graph_stats_host(g.n, g.row_ptr, g.labels) if cost else None
+    plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, code_motion=not nocm, lazy_unbounded=lazy,
+                    cost_stats=stats)
+    if cost:
+        print(f"   {spec}: model cost {plan.model_cost:.3e}, est count {plan.model_count:.3e}, "
+              + plan.describe().split(chr(10))[0], flush=True)
     t = stm.stm_tuning_default(**{k: int(v) for k, v in tk.items()})
     best = 1e9
     try:
