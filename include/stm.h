@@ -352,6 +352,34 @@ stm_status stm_order_optimize(int k, int n_edges, const int32_t* edges, const in
                               const int32_t* restr, uint32_t flags, const stm_graph_stats* stats,
                               int32_t* order_out, double* cost, double* est_count);
 
+/* ---------------------------------------------------------------------------------------
+ * Motif census (many patterns per graph).
+ * ------------------------------------------------------------------------------------- */
+
+/*
+ * stm_motif_catalog -- the connected graphs on k vertices up to isomorphism, 2 <= k <= 6
+ * (1, 2, 6, 21, 112 motifs for k = 2..6), host only.  Motif i has n_edges[i] edges
+ * written as vertex pairs (a < b) to edges[i * k*(k-1) + 2e + {0,1}]; motifs are sorted
+ * by edge count, then by canonical edge mask.  At most `capacity` motifs are written;
+ * *n_motifs receives the full number (call with capacity 0 to size the arrays).
+ * Errors: STM_EUNSUPPORTED (k outside 2..6), STM_EINVAL (NULL n_motifs, NULL arrays
+ * with capacity > 0).
+ */
+stm_status stm_motif_catalog(int k, int capacity, int32_t* n_edges, int32_t* edges, int* n_motifs);
+
+/*
+ * stm_motif_census -- count every motif of stm_motif_catalog(k) in g, in catalog order,
+ * as distinct subgraphs (Grochow-Kellis restrictions).  flags: 0 (edge-induced) or
+ * STM_VERTEX_INDUCED (induced motif frequencies; they sum to the number of connected
+ * induced k-vertex subsets), optionally | STM_NO_CODE_MOTION / STM_LAZY_UNBOUNDED.
+ * One counting launch per motif on `cuda_stream` (synchronous, as stm_match_count_ex);
+ * t may be NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the
+ * catalog size.  Errors: as stm_motif_catalog and stm_match_count_ex; STM_EINVAL for
+ * other flag bits or a short capacity.
+ */
+stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_tuning* t,
+                            void* cuda_stream, int capacity, uint64_t* counts, int* n_motifs);
+
 /* stm_last_error -- thread-local message for the last non-OK status of this thread. */
 const char* stm_last_error(void);
 

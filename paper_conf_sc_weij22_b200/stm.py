@@ -23,7 +23,8 @@ EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_gra
            "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
            "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
            "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error",
-           "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize"]
+           "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize", "stm_motif_catalog",
+           "stm_motif_census"]
 
 
 class StmError(RuntimeError):
@@ -88,6 +89,8 @@ def _load():
         "stm_match_list": [vp, vp, vp, i64, i64, vp, vp, ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
                            ctypes.POINTER(ctypes.c_uint64)],
         "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
+        "stm_motif_catalog": [i32, i32, vp, vp, ctypes.POINTER(i32)],
+        "stm_motif_census": [vp, i32, u32, vp, vp, i32, vp, ctypes.POINTER(i32)],
         "stm_graph_stats_host": [i64, vp, vp, ctypes.POINTER(stm_graph_stats)],
         "stm_order_cost": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
                            ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
@@ -190,6 +193,26 @@ def stm_order_optimize(k: int, edges, labels, restrictions, flags: int,
     _check(lib.stm_order_optimize(k, e.size // 2, _p(e), _p(lb), nr, _p(rs), flags, ctypes.byref(stats), _p(od),
                                   ctypes.byref(c), ctypes.byref(est)))
     return od.tolist(), c.value, est.value
+
+
+def stm_motif_catalog(k: int) -> list:
+    """[(n_edges, [(a, b), ...]), ...] in catalog order."""
+    n = ctypes.c_int()
+    _check(lib.stm_motif_catalog(k, 0, None, None, ctypes.byref(n)))
+    ne = np.zeros(n.value, np.int32)
+    ed = np.zeros(n.value * k * (k - 1), np.int32)
+    _check(lib.stm_motif_catalog(k, n.value, _p(ne), _p(ed), ctypes.byref(n)))
+    s = k * (k - 1)
+    return [[(int(ed[i * s + 2 * e]), int(ed[i * s + 2 * e + 1])) for e in range(ne[i])] for i in range(n.value)]
+
+
+def stm_motif_census(g: int, k: int, flags: int = 0, tuning: Optional[stm_tuning] = None,
+                     stream: Optional[int] = None) -> list:
+    n = ctypes.c_int()
+    cap = 112
+    out = np.zeros(cap, np.uint64)
+    _check(lib.stm_motif_census(g, k, flags, _tp(tuning), stream, cap, _p(out), ctypes.byref(n)))
+    return [int(x) for x in out[: n.value]]
 
 
 def stm_plan_describe(p: int) -> str:

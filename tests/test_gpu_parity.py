@@ -395,3 +395,36 @@ def test_cost_order_counts(rmat_small, name, vi):
     for lab in (None, stmgen.pattern_labels(p.k, 4, 3)):
         plan = stm.Plan(p.k, p.edges, lab, vertex_induced=vi, cost_stats=stats)
         assert stm.count(G, plan) == ocount(g, p, vi, labels=lab)
+
+
+@pytest.mark.parametrize("k", [3, 4, 5])
+@pytest.mark.parametrize("vi", [False, True])
+def test_motif_census(rmat_small, k, vi):
+    """NEXT-3: every motif of the size-k catalog, bit-exact against the oracle."""
+    g, G = rmat_small
+    flags = stm.STM_VERTEX_INDUCED if vi else 0
+    got = stm.stm_motif_census(G.handle, k, flags)
+    cat = stm.stm_motif_catalog(k)
+    assert len(got) == len(cat)
+    for edges, c in zip(cat, got):
+        assert c == oracle.count(g, k, edges, vertex_induced=vi, restrictions=oracle.gk_restrictions(k, edges))
+
+
+def test_motif_census_sums_to_connected_subsets():
+    """Induced motif frequencies partition the connected induced k-vertex subsets
+    (brute force over all k-subsets of a small graph)."""
+    g = stmgen.er(30, 80, 21)
+    G = stm.Graph.from_stmgen(g)
+    adj = [set(g.neighbors(v).tolist()) for v in range(g.n)]
+    for k in (3, 4, 5, 6):
+        want = 0
+        for S in itertools.combinations(range(g.n), k):
+            seen, stack = {S[0]}, [S[0]]
+            while stack:
+                u = stack.pop()
+                for w in S:
+                    if w not in seen and w in adj[u]:
+                        seen.add(w)
+                        stack.append(w)
+            want += len(seen) == k
+        assert sum(stm.stm_motif_census(G.handle, k, stm.STM_VERTEX_INDUCED)) == want
