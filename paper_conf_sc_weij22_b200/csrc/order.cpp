@@ -18,8 +18,10 @@
 //   * cost(pi) = n + sum_{l=1}^{k-1} N(S_l) * work_l,  S_l = {pi[0..l-1]}.
 //
 // The search is exhaustive over connected orders (k <= 8: at most 8! = 40320), and the
-// compiler's greedy order is kept unless another order is strictly cheaper (so cliques
-// and other order-free patterns compile exactly as before).
+// compiler's greedy order is kept unless the best order is predicted at least
+// kMinGain cheaper (so cliques compile exactly as before, and near-ties -- which the
+// model cannot rank, e.g. rotations of a labeled cycle that differ only by label
+// frequencies -- do not move the order; DESIGN.md 8b2 has the measurements).
 #include <algorithm>
 #include <cmath>
 #include <cstring>
@@ -29,6 +31,8 @@
 #include "internal.h"
 
 namespace {
+
+constexpr double kMinGain = 0.10;  // leave the greedy order only for a >= 10% predicted saving
 
 struct Model {
   int k = 0;
@@ -200,8 +204,9 @@ extern "C" stm_status stm_order_optimize(int k, int n_edges, const int32_t* edge
   stm_status st = build_model(k, n_edges, edges, labels, n_restr, restr, flags, stats, &m, &greedy);
   if (st != STM_OK) return st;
   std::vector<int> best = greedy;
-  double best_c, best_e;
-  eval(m, greedy.data(), &best_c, &best_e);
+  double greedy_c, greedy_e;
+  eval(m, greedy.data(), &greedy_c, &greedy_e);
+  double best_c = greedy_c, best_e = greedy_e;
   std::vector<int> p(k);
   for (int i = 0; i < k; ++i) p[i] = i;
   do {
@@ -209,6 +214,7 @@ extern "C" stm_status stm_order_optimize(int k, int n_edges, const int32_t* edge
     if (!eval(m, p.data(), &c, &e)) continue;
     if (c < best_c * (1 - 1e-9)) { best = p; best_c = c; best_e = e; }
   } while (std::next_permutation(p.begin(), p.end()));
+  if (best_c > greedy_c * (1 - kMinGain)) { best = greedy; best_c = greedy_c; best_e = greedy_e; }
   for (int i = 0; i < k; ++i) order_out[i] = best[i];
   if (cost) *cost = best_c;
   if (est_count) *est_count = best_e;
