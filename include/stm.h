@@ -372,13 +372,16 @@ stm_status stm_motif_catalog(int k, int capacity, int32_t* n_edges, int32_t* edg
  * as distinct subgraphs (Grochow-Kellis restrictions).  flags: 0 (edge-induced) or
  * STM_VERTEX_INDUCED (induced motif frequencies; they sum to the number of connected
  * induced k-vertex subsets), optionally | STM_NO_CODE_MOTION / STM_LAZY_UNBOUNDED.
- * One counting launch per motif on `cuda_stream` (synchronous, as stm_match_count_ex);
- * t may be NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the
+ * stats: graph statistics (stm_graph_stats_host) to give each motif its cost-based
+ * order (stm_order_optimize), or NULL for the compiler's greedy order; counts are the
+ * same either way.  One counting launch per motif on `cuda_stream` (synchronous, as
+ * stm_match_count_ex); t may be NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the
  * catalog size.  Errors: as stm_motif_catalog and stm_match_count_ex; STM_EINVAL for
  * other flag bits or a short capacity.
  */
-stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_tuning* t,
-                            void* cuda_stream, int capacity, uint64_t* counts, int* n_motifs);
+stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_graph_stats* stats,
+                            const stm_tuning* t, void* cuda_stream, int capacity, uint64_t* counts,
+                            int* n_motifs);
 
 /* stm_last_error -- thread-local message for the last non-OK status of this thread. */
 const char* stm_last_error(void);

@@ -5,9 +5,9 @@
 // (2, 6, 21, 112 of them for k = 3..6); stm_motif_census counts every one of them on a
 // resident graph with the same counting kernel (one persistent launch per motif on the
 // caller's stream; the graph, its degree-ranked copy and hub bitmaps are built once and
-// shared).  Counts are distinct subgraphs (Grochow-Kellis restrictions); with
-// STM_VERTEX_INDUCED they are the induced motif frequencies, which sum to the number of
-// connected induced k-vertex subsets.
+// shared; given graph statistics, every motif gets its cost-based order).  Counts are
+// distinct subgraphs (Grochow-Kellis restrictions); with STM_VERTEX_INDUCED they are the
+// induced motif frequencies, which sum to the number of connected induced k-vertex subsets.
 #include <algorithm>
 #include <cstring>
 #include <mutex>
@@ -110,8 +110,9 @@ extern "C" stm_status stm_motif_catalog(int k, int capacity, int32_t* n_edges, i
   return STM_OK;
 }
 
-extern "C" stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_tuning* t,
-                                       void* stream, int capacity, uint64_t* counts, int* n_motifs) {
+extern "C" stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_graph_stats* stats,
+                                       const stm_tuning* t, void* stream, int capacity, uint64_t* counts,
+                                       int* n_motifs) {
   if (!g) return stm_fail(STM_EINVAL, "graph is NULL");
   if (k < 2 || k > kMotifKMax) return stm_fail(STM_EUNSUPPORTED, "motif size k=%d outside 2..%d", k, kMotifKMax);
   if (!n_motifs || !counts) return stm_fail(STM_EINVAL, "NULL output");
@@ -123,9 +124,16 @@ extern "C" stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags
   for (size_t i = 0; i < cat.size(); ++i) {
     std::vector<int32_t> e;
     for (auto& pr : cat[i].edges) { e.push_back(pr.first); e.push_back(pr.second); }
+    int32_t order[kMotifKMax];
+    stm_status s = STM_OK;
+    if (stats) {  // cost-based matching order (order.cpp, NEXT-2)
+      s = stm_order_optimize(k, cat[i].n_edges, e.data(), nullptr, 0, nullptr, flags | STM_AUTO_RESTRICT, stats,
+                             order, nullptr, nullptr);
+      if (s != STM_OK) return s;
+    }
     stm_plan* P = nullptr;
-    stm_status s = stm_pattern_compile(k, cat[i].n_edges, e.data(), nullptr, nullptr, 0, nullptr,
-                                       flags | STM_AUTO_RESTRICT, &P);
+    s = stm_pattern_compile(k, cat[i].n_edges, e.data(), nullptr, stats ? order : nullptr, 0, nullptr,
+                            flags | STM_AUTO_RESTRICT, &P);
     if (s != STM_OK) return s;
     uint64_t c = 0;
     s = stm_match_count_ex(g, P, t, nullptr, stream, &c);

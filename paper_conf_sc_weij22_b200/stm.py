@@ -90,7 +90,7 @@ def _load():
                            ctypes.POINTER(ctypes.c_uint64)],
         "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
         "stm_motif_catalog": [i32, i32, vp, vp, ctypes.POINTER(i32)],
-        "stm_motif_census": [vp, i32, u32, vp, vp, i32, vp, ctypes.POINTER(i32)],
+        "stm_motif_census": [vp, i32, u32, vp, vp, vp, i32, vp, ctypes.POINTER(i32)],
         "stm_graph_stats_host": [i64, vp, vp, ctypes.POINTER(stm_graph_stats)],
         "stm_order_cost": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
                            ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
@@ -206,12 +206,13 @@ def stm_motif_catalog(k: int) -> list:
     return [[(int(ed[i * s + 2 * e]), int(ed[i * s + 2 * e + 1])) for e in range(ne[i])] for i in range(n.value)]
 
 
-def stm_motif_census(g: int, k: int, flags: int = 0, tuning: Optional[stm_tuning] = None,
-                     stream: Optional[int] = None) -> list:
+def stm_motif_census(g: int, k: int, flags: int = 0, stats: Optional[stm_graph_stats] = None,
+                     tuning: Optional[stm_tuning] = None, stream: Optional[int] = None) -> list:
     n = ctypes.c_int()
     cap = 112
     out = np.zeros(cap, np.uint64)
-    _check(lib.stm_motif_census(g, k, flags, _tp(tuning), stream, cap, _p(out), ctypes.byref(n)))
+    sp = None if stats is None else ctypes.cast(ctypes.pointer(stats), ctypes.c_void_p)
+    _check(lib.stm_motif_census(g, k, flags, sp, _tp(tuning), stream, cap, _p(out), ctypes.byref(n)))
     return [int(x) for x in out[: n.value]]
 
 

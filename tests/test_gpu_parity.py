@@ -406,6 +406,8 @@ def test_motif_census(rmat_small, k, vi):
     got = stm.stm_motif_census(G.handle, k, flags)
     cat = stm.stm_motif_catalog(k)
     assert len(got) == len(cat)
+    stats = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    assert stm.stm_motif_census(G.handle, k, flags, stats) == got
     for edges, c in zip(cat, got):
         assert c == oracle.count(g, k, edges, vertex_induced=vi, restrictions=oracle.gk_restrictions(k, edges))
 
