@@ -345,7 +345,8 @@ stm_status stm_order_cost(int k, int n_edges, const int32_t* edges, const int32_
 /*
  * stm_order_optimize -- the connected order of minimal model cost (exhaustive over the
  * <= 8! permutations); the compiler's greedy order is kept unless that minimum is at
- * least 10% below the greedy order's cost (near-ties are not ranked by the model).  Writes int32[k] to order_out (caller-owned); cost / est_count as in
+ * least 10% below the greedy order's cost (near-ties are not ranked by the model),
+ * and always for trees (|E| = k - 1; measured).  Writes int32[k] to order_out (caller-owned); cost / est_count as in
  * stm_order_cost (may be NULL).  Errors as stm_order_cost.
  */
 stm_status stm_order_optimize(int k, int n_edges, const int32_t* edges, const int32_t* labels, int n_restr,

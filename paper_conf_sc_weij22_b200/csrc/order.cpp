@@ -21,7 +21,8 @@
 // compiler's greedy order is kept unless the best order is predicted at least
 // kMinGain cheaper (so cliques compile exactly as before, and near-ties -- which the
 // model cannot rank, e.g. rotations of a labeled cycle that differ only by label
-// frequencies -- do not move the order; DESIGN.md 8b2 has the measurements).
+// frequencies -- do not move the order; trees keep it too; DESIGN.md 8b2 has the
+// measurements).
 #include <algorithm>
 #include <cmath>
 #include <cstring>
@@ -36,6 +37,7 @@ constexpr double kMinGain = 0.10;  // leave the greedy order only for a >= 10% p
 
 struct Model {
   int k = 0;
+  int n_edges = 0;
   int adj[STM_KMAX][STM_KMAX] = {};
   double lab_factor[STM_KMAX] = {};
   double ext[1 << STM_KMAX] = {};  // linear extensions of the restriction order on each subset
@@ -106,6 +108,7 @@ stm_status build_model(int k, int n_edges, const int32_t* edges, const int32_t* 
   m->nnz = (double)s->nnz;
   for (int j = 0; j < STM_STATS_MOMENTS; ++j) m->M[j] = s->moment[j];
   for (auto& e : P->edges) m->adj[e.first][e.second] = m->adj[e.second][e.first] = 1;
+  m->n_edges = (int)P->edges.size();
   for (int u = 0; u < k; ++u) {
     m->lab_factor[u] = 1.0;
     if (!P->labels.empty() && P->labels[u] >= 0 && s->n_labels > 0) {
@@ -214,7 +217,11 @@ extern "C" stm_status stm_order_optimize(int k, int n_edges, const int32_t* edge
     if (!eval(m, p.data(), &c, &e)) continue;
     if (c < best_c * (1 - 1e-9)) { best = p; best_c = c; best_e = e; }
   } while (std::next_permutation(p.begin(), p.end()));
-  if (best_c > greedy_c * (1 - kMinGain)) { best = greedy; best_c = greedy_c; best_e = greedy_e; }
+  // Trees: every order has exactly one operand per level, so the model can only rank
+  // where the restriction bounds land, and it ranked that wrong on every tree motif
+  // measured (C1, k = 5/6 vertex-induced: 1.2x-8.3x slower, profiles/r01_census_permotif.log).
+  const bool tree = m.n_edges == k - 1;
+  if (tree || best_c > greedy_c * (1 - kMinGain)) { best = greedy; best_c = greedy_c; best_e = greedy_e; }
   for (int i = 0; i < k; ++i) order_out[i] = best[i];
   if (cost) *cost = best_c;
   if (est_count) *est_count = best_e;

@@ -136,7 +136,7 @@ def test_optimum_over_all_connected_orders(stm, name, vi):
     greedy_order = stm.Plan(p.k, p.edges, vertex_induced=vi, auto_order=True).describe()
     greedy_order = [int(x) for x in greedy_order.split("order=[")[1].split("]")[0].split(",")]
     greedy = costs[tuple(greedy_order)][0]
-    if greedy <= best / 0.9:  # within the 10% hysteresis: the greedy order is kept
+    if greedy <= best / 0.9 or len(p.edges) == p.k - 1:  # hysteresis / trees: the greedy order is kept
         assert order == greedy_order
     else:
         assert cost <= best * (1 + 1e-9)
@@ -154,6 +154,18 @@ def test_near_ties_keep_the_greedy_order(stm):
         order, cost, _ = stm.stm_order_optimize(p.k, p.edges, lab, None, stm.STM_AUTO_RESTRICT, s)
         plan = stm.Plan(p.k, p.edges, lab, auto_order=True)
         assert f"order=[{','.join(map(str, order))}]" in plan.describe()
+
+
+def test_trees_keep_the_greedy_order(stm):
+    g = stmgen.config_graph("c2")
+    s = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    for k in (4, 5, 6):
+        for e in stm.stm_motif_catalog(k):
+            if len(e) != k - 1:
+                continue
+            order, _, _ = stm.stm_order_optimize(k, e, None, None, stm.STM_AUTO_RESTRICT | stm.STM_VERTEX_INDUCED, s)
+            plan = stm.Plan(k, e, vertex_induced=True, auto_order=True)
+            assert f"order=[{','.join(map(str, order))}]" in plan.describe()
 
 
 @pytest.mark.parametrize("name", ["triangle", "k4", "k5", "k6", "k8"])

@@ -39,8 +39,12 @@ for spec in sys.argv[1:]:
         if best == gr or bc >= gc * (1 - 1e-9):
             continue
         pc = stm.Plan(k, e, vertex_induced=vi, order=best)
-        c1, t1 = best_of(G, pg)
-        c2, t2 = best_of(G, pc)
+        try:
+            c1, t1 = best_of(G, pg)
+            c2, t2 = best_of(G, pc)
+        except stm.StmError as ex:
+            print(f"{spec} motif {i:3d} pred {bc / gc:.3f} ERR {ex}", flush=True)
+            continue
         assert c1 == c2
         print(f"{spec} motif {i:3d} pred {bc / gc:.3f} measured {t2 / t1:.3f}  greedy {t1 * 1e3:8.2f} ms  "
               f"cost {t2 * 1e3:8.2f} ms  count {c1}", flush=True)
