@@ -14,8 +14,10 @@
 //     of linear extensions of the restriction partial order restricted to S);
 //   * extending one level-l prefix costs the summed expected neighbour-list lengths of
 //     the set operands: the backward neighbours b of pi[l] (and, vertex-induced, the
-//     backward non-neighbours), E[w(f(b))] = M_{j+1} / M_j with j = deg_{H_l}(b);
-//   * cost(pi) = n + sum_{l=1}^{k-1} N(S_l) * work_l,  S_l = {pi[0..l-1]}.
+//     backward non-neighbours), E[w(f(b))] = M_{j+1} / M_j with j = deg_{H_l}(b) --
+//     except with a single operand, where the candidates are a bounded view of one row
+//     (cost 1 + log2(1 + E[w])); inner-level candidates are then visited one by one;
+//   * cost(pi) = n + sum_{l=1}^{k-1} N(S_l) * work_l + sum_{l=2}^{k-1} N(S_l).
 //
 // The search is exhaustive over connected orders (k <= 8: at most 8! = 40320), and the
 // compiler's greedy order is kept unless the best order is predicted at least
@@ -54,6 +56,7 @@ bool eval(const Model& m, const int* pi, double* cost, double* est) {
   int degH[STM_KMAX] = {};  // degree of each placed pattern vertex inside H_l
   int edgesH = 0;
   double N = 0;
+  bool visit_next = false;
   auto count_of = [&](unsigned set) {  // N(S) from the closed form above
     if (m.nnz <= 0) return 0.0;
     double v = 1.0;
@@ -71,19 +74,28 @@ bool eval(const Model& m, const int* pi, double* cost, double* est) {
     if (l > 0) {
       bool con = false;
       double work = 0;
+      int ops = 0;
       for (int b = 0; b < k; ++b) {
         if (!(S >> b & 1)) continue;
         const bool nb = m.adj[u][b];
         con |= nb;
-        if (nb || m.vi) work += m.M[degH[b]] > 0 ? m.M[degH[b] + 1] / m.M[degH[b]] : 0;
+        if (nb || m.vi) {
+          work += m.M[degH[b]] > 0 ? m.M[degH[b] + 1] / m.M[degH[b]] : 0;
+          ++ops;
+        }
       }
       if (!con) return false;
+      // One operand: the candidates are a bounded view of one row (no set operation),
+      // a binary search for the bounds; at the last level its size is the count.
+      if (ops == 1) work = 1 + std::log2(1 + work);
       c += N * work;
+      visit_next = l < k - 1;  // candidates of inner levels are iterated one by one
       for (int b = 0; b < k; ++b)
         if ((S >> b & 1) && m.adj[u][b]) { ++degH[b]; ++degH[u]; ++edgesH; }
     }
     S |= 1u << u;
     N = count_of(S);
+    if (visit_next) c += N;
   }
   *cost = c;
   *est = N;
