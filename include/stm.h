@@ -49,7 +49,8 @@ typedef enum {
   STM_ENOMEM = 2,        /* host or device allocation failed */
   STM_ECUDA = 3,         /* a CUDA runtime call failed */
   STM_EUNSUPPORTED = 4,  /* valid request outside this build's limits (k > 8, > 255 graph labels, ...) */
-  STM_EOVERFLOW = 5      /* device scratch / stack capacity exceeded: no count produced */
+  STM_EOVERFLOW = 5,     /* device scratch / stack capacity exceeded: no count produced */
+  STM_ETIMEOUT = 6       /* the launch ran longer than stm_tuning.watchdog_ms and was aborted: no count */
 } stm_status;
 
 typedef struct stm_graph stm_graph; /* opaque, device-resident, immutable */
@@ -82,7 +83,9 @@ enum { STM_K_MAX = 8 };
  *   device   CUDA device ordinal.
  *   out      receives the handle.
  * Errors: STM_EINVAL for any CSR violation above (the full check is O(m log d)
- * on the host), STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED.
+ * on the host), STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED (> 255 labels, or
+ * row_ptr[n] >= 2^32 adjacency entries: the kernel's packed per-vertex records hold
+ * 32-bit row starts).
  */
 stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                           const int32_t* labels, int device, stm_graph** out);
@@ -181,6 +184,15 @@ typedef struct stm_tuning {
   int32_t narrow_split;      /* 0 = narrow neighbour lists to restriction bounds with the per-vertex split
                              out_start[v] (first neighbour > v, built at load); 1 = binary search only.
                              Speed only.  Default 0. */
+  int32_t watchdog_ms;    /* failure detection: a launch still running after this many milliseconds of
+                             device time aborts itself and the call reports STM_ETIMEOUT (never a partial
+                             count; the async call reports it in stm_async_result.status).  0 = off.
+                             Default 0. */
+  int32_t backoff_max;    /* idle warps sleep up to 32 << backoff_max ns between failed steal attempts
+                             (0..12); 0 = auto (8, measured).  Speed only. */
+  int32_t carveout_pct;   /* shared-memory carveout of the unified L1/shared array in percent: 0 = auto
+                             (just enough for the resident DFS stacks, rest to L1), -1 = driver default,
+                             else 1..100.  Speed only. */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -221,12 +233,50 @@ stm_status stm_match_count_ex(const stm_graph* g, const stm_plan* p, const stm_t
                               const stm_shard* shard, void* cuda_stream, uint64_t* count);
 
 /*
- * stm_match_count_async -- enqueue the kernel and leave the count in DEVICE
- * memory (d_count: one uint64, overwritten) without synchronising.  Used by the
- * benchmark and the multi-GPU layer (the all-reduce then runs on d_count).
+ * Result record of an asynchronous count, written in DEVICE memory by the launch
+ * itself (the last block to finish writes it; no extra copy is enqueued).
+ */
+typedef struct stm_async_result {
+  uint64_t count;        /* the (partial, with a shard) count mod 2^64; meaningful only if status == 0 */
+  uint64_t status;       /* 0 = OK, else the stm_status the synchronous call would have returned
+                            (STM_EOVERFLOW, STM_ETIMEOUT): the count must not be used */
+  uint64_t chunks;       /* root chunks this launch took from all cursors */
+  uint64_t peer_chunks;  /* ... of which from peer ranks' cursors (cross-GPU stealing) */
+} stm_async_result;
+
+/*
+ * stm_match_count_async -- enqueue the kernel on cuda_stream and return without
+ * synchronising; the launch overwrites *d_result (device memory, 32 bytes, 8-byte
+ * aligned) when it completes.  Used by the benchmark and the multi-GPU layer: the
+ * all-reduce runs on d_result->count and the caller checks d_result->status
+ * (summed statuses are non-zero iff some rank failed).  Host-side argument errors
+ * are returned immediately; device-side failures only through d_result->status.
  */
 stm_status stm_match_count_async(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
-                                 const stm_shard* shard, void* cuda_stream, uint64_t* d_count);
+                                 const stm_shard* shard, void* cuda_stream, stm_async_result* d_result);
+
+/*
+ * Chunk cursors shared across processes (multi-GPU layer, PAPER.md:164 + north_star's
+ * cross-GPU stealing): every rank allocates its cursors on its own GPU and exports a
+ * CUDA IPC handle; every peer maps it, so a kernel whose own cursor is exhausted takes
+ * root chunks from a peer's cursor with atomics over NVLink (or, for ranks sharing one
+ * GPU, in the same HBM).
+ *   stm_cursors_alloc  n_slots zeroed uint64 cursors, 64 bytes apart (slot s at
+ *                      d_base + 8*s words), on `device`; *ipc_handle receives
+ *                      STM_IPC_HANDLE_BYTES bytes to send to the peers.
+ *   stm_cursors_open   map a peer's handle into this process (on `device`); the peer's
+ *                      cursors must stay allocated until stm_cursors_close.
+ *   stm_cursors_close / stm_cursors_free  unmap / release.
+ * Errors: STM_EINVAL (NULL out, n_slots < 1, bad device), STM_ECUDA (IPC unsupported).
+ */
+enum { STM_IPC_HANDLE_BYTES = 64 };
+stm_status stm_cursors_alloc(int device, int n_slots, uint64_t** d_base, void* ipc_handle);
+stm_status stm_cursors_open(int device, const void* ipc_handle, uint64_t** d_peer_base);
+stm_status stm_cursors_close(int device, uint64_t* d_peer_base);
+/* stm_cursors_reset -- zero n_slots cursors from slot first_slot of THIS process's own
+   allocation, in stream order on cuda_stream (cudaMemsetAsync). */
+stm_status stm_cursors_reset(int device, uint64_t* d_base, int first_slot, int n_slots, void* cuda_stream);
+stm_status stm_cursors_free(int device, uint64_t* d_base);
 
 /*
  * stm_match_count_per_root -- localisation build: host uint64[n] receives, for every
@@ -284,6 +334,7 @@ typedef struct stm_launch_info {
   int64_t hubs;            /* vertices with a hub adjacency bitmap in the counted numbering */
   int32_t variant;         /* kernel variant launched (stm_tuning.occupancy: 1 or 2) */
   int32_t unroll;          /* unroll factor used */
+  int64_t peer_chunks;     /* root chunks taken from peer ranks' cursors (shard launches); synchronous calls only */
 } stm_launch_info;
 
 stm_status stm_last_launch(stm_launch_info* info);
@@ -327,6 +378,14 @@ typedef struct stm_graph_stats {
  */
 stm_status stm_graph_stats_host(int64_t n, const int64_t* row_ptr, const int32_t* labels,
                                 stm_graph_stats* out);
+
+/*
+ * stm_graph_get_stats -- the statistics of a loaded graph (computed by stm_graph_load /
+ * stm_graph_load_device exactly as stm_graph_stats_host does), so callers get the
+ * cost-based order without keeping host arrays: stm_motif_census uses them by default.
+ * Errors: STM_EINVAL (NULL), STM_EUNSUPPORTED (graph with > 256 distinct labels).
+ */
+stm_status stm_graph_get_stats(const stm_graph* g, stm_graph_stats* out);
 
 /*
  * stm_order_cost -- model cost of matching `order` (int32[k], a connected permutation)
@@ -374,8 +433,8 @@ stm_status stm_motif_catalog(int k, int capacity, int32_t* n_edges, int32_t* edg
  * STM_VERTEX_INDUCED (induced motif frequencies; they sum to the number of connected
  * induced k-vertex subsets), optionally | STM_NO_CODE_MOTION / STM_LAZY_UNBOUNDED.
  * stats: graph statistics (stm_graph_stats_host) to give each motif its cost-based
- * order (stm_order_optimize), or NULL for the compiler's greedy order; counts are the
- * same either way.  One counting launch per motif on `cuda_stream` (synchronous, as
+ * order (stm_order_optimize), or NULL for the graph's own statistics (stm_graph_get_stats);
+ * flags | STM_AUTO_ORDER keeps the compiler's greedy order.  Counts are the same either way.  One counting launch per motif on `cuda_stream` (synchronous, as
  * stm_match_count_ex); t may be NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the
  * catalog size.  Errors: as stm_motif_catalog and stm_match_count_ex; STM_EINVAL for
  * other flag bits or a short capacity.

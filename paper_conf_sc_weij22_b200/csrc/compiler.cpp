@@ -104,6 +104,11 @@ static void build_describe(stm_plan* P) {
            op.c_str(), lab(f.lab).c_str(), fmt_mask(f.lo).c_str(), fmt_mask(f.hi).c_str(),
            fmt_mask(f.excl).c_str());
   s += buf;
+  s += "need=[";
+  for (int l = 1; l < D.k; ++l) s += (l > 1 ? "," : "") + std::to_string(D.need[l]);
+  s += "] pretest=[";
+  for (int l = 1; l < D.k; ++l) s += (l > 1 ? "," : "") + std::to_string(D.pretest[l]);
+  s += "]\n";
   snprintf(buf, sizeof buf, "scratch_words_per_warp_per_cap=%d\n", D.n_nodes);
   s += buf;
   P->describe = s;
@@ -439,6 +444,51 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     D.filt[l].lo = (uint8_t)reduce_lo(lo_pos[l]);
     D.filt[l].hi = (uint8_t)reduce_hi(hi_pos[l]);
     D.filt[l].excl = (uint8_t)excl[l];
+  }
+
+  // ---- candidate-set pruning (plan.h need / pretest).  v_m (m > l) is necessarily an
+  // element of level l's candidate set C_l = S_l ∩ filter_l when (i) m's candidate
+  // source is a subset of S_l (S_l itself, a node whose operand chain passes through
+  // S_l, or a chain starting at the same raw list) and (ii) the pattern forces v_m
+  // through filter_l: every bound of level l holds for pi[m] by the restriction closure
+  // and the label matches.  Injectivity makes v_l and those v_m distinct elements of C_l.
+  {
+    auto chain_has = [&](StmSrc t, StmSrc s) {  // t ⊆ s through t's operand chain
+      for (;;) {
+        if (t.kind == s.kind && t.idx == s.idx) return true;
+        if (t.kind == STM_SRC_RAW) return false;
+        const StmNode& nd = D.nodes[t.idx];
+        t.kind = nd.a_kind;
+        t.idx = nd.a;
+      }
+    };
+    auto src_of = [&](int m) -> StmSrc {  // a set containing every candidate of level m
+      return m == k - 1 ? D.cnt_a : D.cand[m];
+    };
+    for (int l = 1; l < k; ++l) {
+      int need = 1;
+      const StmSrc s = src_of(l);
+      const unsigned lm = labmask(l);
+      for (int m = l + 1; m < k; ++m) {
+        if (!chain_has(src_of(m), s)) continue;
+        if (lm != STM_LAB_ANY && labmask(m) != lm) continue;
+        bool forced = true;
+        for (int j = 0; j < l && forced; ++j) {
+          if ((lo_pos[l] >> j & 1) && !less[pi[j]][pi[m]]) forced = false;
+          if ((hi_pos[l] >> j & 1) && !less[pi[m]][pi[j]]) forced = false;
+        }
+        if (forced) ++need;
+      }
+      D.need[l] = (int8_t)need;
+      // pre-test: unbounded stage-0 node of level l feeding a bounded consumer
+      D.pretest[l] = 0;
+      if (l >= 2 && l < k - 1 && D.cand[l].kind == STM_SRC_NODE) {
+        const StmNode& nd = D.nodes[D.cand[l].idx];
+        if (nd.level == l && nd.stage == 0 && (D.filt[l].lo | D.filt[l].hi) &&
+            ((D.filt[l].lo & ~nd.lo) | (D.filt[l].hi & ~nd.hi)))
+          D.pretest[l] = 1;
+      }
+    }
   }
   build_describe(P);
   *out = P;

@@ -64,9 +64,6 @@
 #else
 #define HDR_SYNC() ((void)0)
 #endif
-#ifndef STM_DRIVE_RATIO
-#define STM_DRIVE_RATIO 0  // 1: compile in the drive_ratio operand choice (measured slower; A/B builds)
-#endif
 #ifndef STM_GATHER_SLOW_NOINLINE
 #define STM_GATHER_SLOW_NOINLINE 0  // 1: the per-candidate admission path out of line (A/B)
 #endif
@@ -77,9 +74,6 @@
 #endif
 #ifndef STM_OCC_MAXT
 #define STM_OCC_MAXT 1536   // __launch_bounds__ of the high-occupancy variant (40 registers)
-#endif
-#ifndef STM_ILP2
-#define STM_ILP2 0          // 1: element loop handles two 32-element slices per iteration (probe ILP)
 #endif
 #ifndef STM_INSTR
 #define STM_INSTR 0         // 1: the instrumented build (kernel_instr.cu): algorithmic-byte / idle counters
@@ -93,6 +87,9 @@
 #define STM_SYM(x) x##_list
 #else
 #define STM_SYM(x) x
+#endif
+#ifndef STM_DEBUG
+#define STM_DEBUG 0         // 1: watchdog state dumps (printf)
 #endif
 #ifndef STM_PROFILE
 #define STM_PROFILE 0       // 1: per-phase clock64() buckets (stm_last_profile); A/B builds only
@@ -109,10 +106,6 @@
 #define PROF_BEGIN(id)
 #define PROF_END(id, items)
 #endif
-#ifndef STM_WITH_HASH
-#define STM_WITH_HASH 0  // per-warp shared-memory hash sets (stm_tuning.hash_slots): measured slower, off
-#endif
-#define HT_MIN 16
 
 namespace {
 
@@ -123,7 +116,13 @@ struct WarpHdr {
   int nsib[STM_KMAX], cur[STM_KMAX], it[STM_KMAX], end[STM_KMAX];
   int used[STM_MAX_NODES];    // words used in each node region by the frame being built
   int stage_c[32], stage_u[32];
-  unsigned lgen[STM_KMAX + 1];  // per-level generation of the arena set nodes
+  // per-warp scheduler state kept here (not in registers) so that the cold, out-of-line
+  // work-acquisition functions need no reference to the warp's register state
+  unsigned exhausted;         // cursors known to be exhausted (bit per rank)
+  unsigned donate_tick;
+  int steal_fails;
+  int pad0;
+  long long first_dry;        // STM_PROFILE: clock64() when the root cursors were first seen exhausted
 };
 
 struct BlockHdr {
@@ -140,6 +139,11 @@ __host__ __device__ inline int warp_bytes(int k, int n_nodes, int ht_slots) {
   return (b + 15) & ~15;
 }
 
+// The warp's view of the launch: pointers into the grid-constant parameters and the
+// warp's shared-memory stack.  It is rebuilt from threadIdx by make_w() wherever it is
+// needed and never passed by reference to an out-of-line function, so that it stays in
+// registers (an escaping W lives in local memory and turns every stack-header access
+// into a generic load).
 struct W {
   const StmKParams* kp;
   const StmPlan* P;
@@ -150,23 +154,58 @@ struct W {
   BlockHdr* bh;
   int* arena;
   int lane, wid;
-  unsigned exhausted;  // cursors known to be exhausted (bit per rank)
   unsigned long long cnt;
-  unsigned gather_calls;
-  unsigned donate_tick;
-  int steal_fails;
   unsigned long long wbytes, wmerge, wjobs;  // per-lane instrumentation partials
   unsigned long long idle_cyc;               // cycles in acquire_work (instrumented launches)
 #if STM_PROFILE
   unsigned long long prof_cyc[STM_PROF_N], prof_cnt[STM_PROF_N], prof_items[STM_PROF_N];
-  long long first_dry;  // clock64() when the root cursors were first seen exhausted
 #endif
-  int* ht;                          // shared-memory hash set (HT_SLOTS ints)
-  unsigned ht_mask;
-  unsigned long long ht_ptr;        // key of the hashed operand
-  int ht_len;
-  unsigned ht_gen;                  // lgen of the hashed node's level when it was hashed
 };
+
+extern __shared__ __align__(16) unsigned char stm_smem[];
+
+__device__ __forceinline__ W make_w(const StmKParams& kp) {
+  const StmPlan& P = kp.plan;
+  W w;
+  w.kp = &kp;
+  w.P = &P;
+  w.lane = threadIdx.x & 31;
+  w.wid = threadIdx.x >> 5;
+  const int wb = warp_bytes(P.k, P.n_nodes, kp.ht_slots);
+  unsigned char* wbase = stm_smem + sizeof(BlockHdr) + (size_t)w.wid * wb;
+  w.bh = (BlockHdr*)stm_smem;
+  w.h = (volatile WarpHdr*)wbase;
+  w.sib = (volatile int*)(wbase + sizeof(WarpHdr));
+  w.noff = (int*)(wbase + sizeof(WarpHdr) + P.k * STM_RMAX * 4);
+  w.nsz = w.noff + P.n_nodes * STM_UMAX;
+  const long long gw = (long long)blockIdx.x * kp.block_warps + w.wid;
+  w.arena = kp.arena + (size_t)gw * (size_t)P.n_nodes * (size_t)kp.cap;
+  w.cnt = 0;
+  w.wbytes = w.wmerge = w.wjobs = 0;
+  w.idle_cyc = 0;
+#if STM_PROFILE
+  for (int i = 0; i < STM_PROF_N; ++i) w.prof_cyc[i] = w.prof_cnt[i] = w.prof_items[i] = 0;
+#endif
+  return w;
+}
+
+// instrumented builds: add a W's per-lane algorithmic-byte partials to the launch totals
+__device__ __forceinline__ void flush_instr(W& w) {
+  if (STM_INSTR && w.kp->count_bytes) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      w.wbytes += __shfl_xor_sync(FULLMASK, w.wbytes, o);
+      w.wmerge += __shfl_xor_sync(FULLMASK, w.wmerge, o);
+      w.wjobs += __shfl_xor_sync(FULLMASK, w.wjobs, o);
+    }
+    if (w.lane == 0) {
+      atomicAdd(&w.kp->work->alg_bytes, w.wbytes);
+      atomicAdd(&w.kp->work->merge_bytes, w.wmerge);
+      atomicAdd(&w.kp->work->n_jobs, w.wjobs);
+    }
+    w.wbytes = w.wmerge = w.wjobs = 0;
+  }
+}
 
 #define SIB(w, l, u) ((w).sib[(l) * STM_RMAX + (u)])
 #define NOFF(w, s, u) ((w).noff[(s) * STM_UMAX + (u)])
@@ -200,33 +239,17 @@ __device__ __forceinline__ bool member(const int* __restrict__ a, int n, int x) 
   return *base == x;
 }
 
-// Two independent membership searches interleaved (element-loop ILP): the dependent
-// probe chains of two elements overlap instead of running back to back.
-__device__ __forceinline__ void member2(const int* __restrict__ pa, int na, int xa, const int* __restrict__ pb,
-                                        int nb, int xb, bool& fa, bool& fb) {
-  const int* ba = pa;
-  const int* bb = pb;
-  int ra = na, rb = nb;
-  while (ra > 1 || rb > 1) {
-    if (ra > 1) { const int h = ra >> 1; ba = (ba[h] <= xa) ? ba + h : ba; ra -= h; }
-    if (rb > 1) { const int h = rb >> 1; bb = (bb[h] <= xb) ? bb + h : bb; rb -= h; }
-  }
-  fa = na > 0 && *ba == xa;
-  fb = nb > 0 && *bb == xb;
-}
-
+// Packed per-vertex record (StmKParams::vrec, built at the first launch per numbering and
+// hub set): x = row start in col_idx, y = degree, z = out_start (index of the first
+// neighbour > v, -1 = unknown), w = hub bitmap slot (-1 = none) -- one 16-byte load
+// instead of row_ptr[v], row_ptr[v+1], out_start[v] and hub_slot[v] from four arrays.
+__device__ __forceinline__ int4 vrec(const W& w, int v) { return __ldg(w.kp->vrec + v); }
 __device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) {
-  long long b = w.kp->row_ptr[v], e = w.kp->row_ptr[v + 1];
-  p = w.kp->col_idx + b;
-  len = (int)(e - b);
+  const int4 r = vrec(w, v);
+  p = w.kp->col_idx + (unsigned)r.x;
+  len = r.y;
 }
-// bitmap slot of v's neighbour list, -1 when v has none
-__device__ __forceinline__ int hslot(const W& w, int v) {
-  return w.kp->hub_slot ? w.kp->hub_slot[v] : -1;
-}
-__device__ __forceinline__ int degree(const W& w, int v) {
-  return (int)(w.kp->row_ptr[v + 1] - w.kp->row_ptr[v]);
-}
+__device__ __forceinline__ int degree(const W& w, int v) { return vrec(w, v).y; }
 
 // value of v_j in the context "frame F, sibling u, candidate c of level F"
 __device__ __forceinline__ int pval(const W& w, int j, int F, int u, int c) {
@@ -263,43 +286,6 @@ __device__ __forceinline__ bool labok(const W& w, int x, unsigned lab) {
 }
 
 // ----------------------------------------------------------------------------
-// Per-warp shared-memory hash set of one sorted operand (B200 design choice, see
-// DESIGN.md "Kernel"): when every job of a combined operation shares an operand
-// (a set of the current DFS path, e.g. N(v0) for all level-2 jobs of a root), it
-// is hashed once into the warp's shared-memory table and every membership probe
-// becomes ~1 shared-memory load instead of a binary search through L1/L2.  The
-// table stays valid while the same operand is reused by later operations.
-// ----------------------------------------------------------------------------
-__device__ __forceinline__ unsigned ht_hash(int x, unsigned mask) {
-  return (((unsigned)x * 0x9E3779B1u) >> 7) & mask;
-}
-
-__device__ __noinline__ void ht_build(W& w, const int* a, int n) {
-  unsigned size = 64;
-  while (size < 2u * (unsigned)n) size <<= 1;
-  const unsigned mask = size - 1;
-  for (unsigned i = w.lane; i < size; i += 32) w.ht[i] = -1;
-  __syncwarp();
-  for (int i = w.lane; i < n; i += 32) {
-    const int x = a[i];
-    unsigned h = ht_hash(x, mask);
-    while (atomicCAS(&w.ht[h], -1, x) != -1) h = (h + 1) & mask;
-  }
-  __syncwarp();
-  w.ht_mask = mask;
-}
-
-__device__ __forceinline__ bool ht_has(const int* ht, unsigned mask, int x) {
-  unsigned h = ht_hash(x, mask);
-  for (;;) {
-    const int v = ht[h];
-    if (v == x) return true;
-    if (v < 0) return false;
-    h = (h + 1) & mask;
-  }
-}
-
-// ----------------------------------------------------------------------------
 // Flattened multi-job set operation (Fig. 8).  Lane j < njobs owns job j.
 // ----------------------------------------------------------------------------
 struct Job {
@@ -323,13 +309,12 @@ __device__ __forceinline__ void narrow(const int*& p, int& n, int lo, int hi) {
 }
 
 // Narrow the CSR row p[0..n) of vertex v to the open interval (lo, hi) at job
-// construction.  out_start[v] splits the sorted row at v (p[0..s) < v < p[s..n)),
-// so the bound lo = v (the common case v_{l-1} < w of a restriction chain) costs one
-// load and every other bound searches only one side of the split.
-__device__ __forceinline__ void narrow_row(const W& w, int v, const int*& p, int& n, int lo, int hi) {
+// construction.  The split s = out_start[v] cuts the sorted row at v (p[0..s) < v <
+// p[s..n)), so the bound lo = v (the common case v_{l-1} < w of a restriction chain)
+// costs nothing and every other bound searches only one side of the split.
+__device__ __forceinline__ void narrow_split(int v, int s, const int*& p, int& n, int lo, int hi) {
   if (lo < 0 && hi == INT_MAX) return;
-  if (!w.kp->out_start) { narrow(p, n, lo, hi); return; }
-  const int s = w.kp->out_start[v];
+  if (s < 0) { narrow(p, n, lo, hi); return; }
   const bool big = n > 16;
   int b = 0, e = n;
   if (lo >= v) { b = s; if (lo > v && big) b += lbound(p + s, n - s, lo + 1); }
@@ -342,12 +327,23 @@ __device__ __forceinline__ void narrow_row(const W& w, int v, const int*& p, int
   n = e - b;
 }
 
+// N(v) from its packed record, narrowed to (lo, hi); hub receives v's bitmap slot
+__device__ __forceinline__ void row_narrow(const W& w, int v, const int*& p, int& n, int& hub, int lo, int hi) {
+  const int4 r = vrec(w, v);
+  p = w.kp->col_idx + (unsigned)r.x;
+  n = r.y;
+  hub = r.w;
+  narrow_split(v, w.kp->split ? r.z : -1, p, n, lo, hi);
+}
+
 __device__ __forceinline__ int log2c(int n) { return 32 - __clz(n); }  // ceil(log2(n+1))
 
 // Returns the (warp-uniform) number of kept elements summed over all jobs when
-// counting; in materialise mode *outc (lane j) receives job j's output size.
+// counting; in materialise mode *outc (lane j) receives job j's output size.  probe:
+// count mode for the candidate-set pre-test (plan.h pretest) -- *outc (lane j) receives
+// job j's count, with no exclusion correction, per-root attribution or listing.
 __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool count_mode, int F,
-                                                    unsigned excl, int* outc_lane) {
+                                                    unsigned excl, int* outc_lane, bool probe = false) {
   const int lane = w.lane;
   PROF_BEGIN(10)
   const bool mine = lane < njobs;
@@ -358,79 +354,21 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   int bn = (mine && J.B) ? J.blen : 0;
   // CSR-row operands were narrowed at job construction (narrow_row); arena sets here
   if (mine && J.a_node) narrow(An, an, J.lo, J.hi);
-  // ---- shared operand -> shared-memory hash set
-  const unsigned long long a0 = __shfl_sync(FULLMASK, (unsigned long long)J.A, 0);
-  const unsigned long long b0 = __shfl_sync(FULLMASK, (unsigned long long)J.B, 0);
-  const int al0 = __shfl_sync(FULLMASK, J.alen, 0), bl0 = __shfl_sync(FULLMASK, J.blen, 0);
-  const int op0 = __shfl_sync(FULLMASK, J.op, 0);
-  const bool sameA = __all_sync(FULLMASK, !mine || ((unsigned long long)J.A == a0 && J.alen == al0 && J.op == STM_OP_AND));
-  const bool sameB = __all_sync(FULLMASK, !mine || ((unsigned long long)J.B == b0 && J.blen == bl0 && J.B != nullptr));
-  int hmode = 0;  // 1: A hashed (drive B), 2: B hashed (drive A)
-  const int* hp = nullptr;
-  int hn = 0;
-  int hnode = 0;
-  const int ht_max = w.kp->ht_slots / 2;
-  if (STM_WITH_HASH && sameA && al0 >= HT_MIN && al0 <= ht_max && b0 != 0ull) {  // (warp-uniform: lane 0 owns a job)
-    hmode = 1; hp = (const int*)a0; hn = al0; hnode = __shfl_sync(FULLMASK, J.a_node, 0);
-  } else if (STM_WITH_HASH && sameB && bl0 >= HT_MIN && bl0 <= ht_max) {
-    hmode = 2; hp = (const int*)b0; hn = bl0;
-  }
-  if (hmode) {
-    const unsigned g = hnode ? w.h->lgen[hnode - 1] : 0u;
-    const bool cached = (unsigned long long)hp == w.ht_ptr && hn == w.ht_len && w.ht_gen == g;
-    if (!cached) {
-      // build only if the probes it saves outweigh the build (~ table size + 2n lane-ops)
-      int save = 0;
-      if (mine) {
-        const int dh = hmode == 1 ? bn : an;  // driven elements in hash mode
-        int d, pl;
-        if (J.op == STM_OP_AND) { d = min(an, bn); pl = max(an, bn); } else { d = an; pl = bn; }
-        save = max(0, d * (log2c(pl) + 1) * 4 - dh * 2);
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) save += __shfl_xor_sync(FULLMASK, save, o);
-      if (save > 4 * hn + 128) {
-        ht_build(w, hp, hn);
-        w.ht_ptr = (unsigned long long)hp;
-        w.ht_len = hn;
-        w.ht_gen = g;
-      } else {
-        hmode = 0;
-      }
-    }
-  }
-  // ---- per-job driving side: 0 = binary search, 1 = hash probe
+  // ---- per-job driving side: for an intersection the shorter (bound-narrowed) operand
+  // drives and the longer one is probed
   const int* D = An;
   const int* Pp = Bn;
-  int dlen = an, plen = bn, use_h = 0;
-  // every job's A ends at the same address: one shared (suffix of a) list, hot in L1
-  bool hotA = false;
-  if (STM_DRIVE_RATIO && w.kp->drive_ratio > 1) {
-    const unsigned long long aend = mine ? (unsigned long long)(J.A + J.alen) : 0ull;
-    const unsigned long long aend0 = __shfl_sync(FULLMASK, aend, 0);
-    hotA = __all_sync(FULLMASK, !mine || aend == aend0);
-  }
+  int dlen = an, plen = bn;
   int pslot = -1;  // bitmap slot of the probed operand
   if (mine) {
     pslot = J.bbm;
-    // drive the shorter operand; with a warp-shared (L1-hot) A, drive B while it is at
-    // most drive_ratio times longer: coalesced reads of B and L1-resident probes into A
-    // instead of DRAM-missing probes into B (stm_tuning.drive_ratio)
-    if (J.op == STM_OP_AND && (bn < an || (hotA && bn <= an * w.kp->drive_ratio))) {
+    if (J.op == STM_OP_AND && bn < an) {
       D = Bn; dlen = bn; Pp = An; plen = an; pslot = J.abm;
     }
     if (!J.B) { Pp = nullptr; plen = 0; pslot = -1; }
     // a probed hub row is tested in its bitmap: one word per element instead of
     // ceil(log2 |P|) dependent loads (the driving element already lies in (lo, hi))
     if (pslot >= 0) Pp = (const int*)(w.kp->bitmaps + (size_t)pslot * (size_t)w.kp->bm_words);
-    if (hmode) {
-      const int dh = hmode == 1 ? bn : an;
-      if (dh * 2 <= dlen * (log2c(plen) + 1) * 4) {
-        use_h = 1;
-        pslot = -1;
-        if (hmode == 1) { D = Bn; dlen = bn; } else { D = An; dlen = an; }
-      }
-    }
   }
   if (STM_INSTR && w.kp->count_bytes && mine) {
     // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below),
@@ -451,84 +389,13 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   }
   const int total = __shfl_sync(FULLMASK, incl, 31);
   const int start = incl - dlen;
-  const int flags = (Pp != nullptr ? 1 : 0) | (use_h ? 2 : 0) | (J.op == STM_OP_DIFF ? 4 : 0) | (pslot >= 0 ? 8 : 0);
-  const int* const ht = w.ht;
-  const unsigned htmask = w.ht_mask;
+  const int flags = (Pp != nullptr ? 1 : 0) | (J.op == STM_OP_DIFF ? 4 : 0) | (pslot >= 0 ? 8 : 0);
   const uint8_t* const glabels = w.kp->labels;
   const unsigned char* const l2s = w.bh->lab2slot;
   int outc = 0;
   unsigned long long jc = 0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
                            Oll = (unsigned long long)J.out;
-#if STM_ILP2 && !STM_LIST
-  // two 32-element slices per iteration: slice h covers elements e0 + 32h + lane
-  for (int e0 = 0; e0 < total; e0 += 64) {
-    int j[2], x[2], fjs[2];
-    const int* Pjs[2];
-    int pls[2];
-    bool keep[2], need[2];
-    unsigned labjs[2];
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int e = e0 + 32 * h + lane;
-      int jj = 0;
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1) {
-        int v = __shfl_sync(FULLMASK, incl, jj + step - 1);
-        if (v <= e) jj += step;
-      }
-      j[h] = jj;
-      const bool valid = e < total;
-      const int* Dj = (const int*)__shfl_sync(FULLMASK, Dll, jj);
-      Pjs[h] = (const int*)__shfl_sync(FULLMASK, Pll, jj);
-      const int sj = __shfl_sync(FULLMASK, start, jj);
-      pls[h] = __shfl_sync(FULLMASK, plen, jj);
-      fjs[h] = __shfl_sync(FULLMASK, flags, jj);
-      const int loj = __shfl_sync(FULLMASK, J.lo, jj);
-      const int hij = __shfl_sync(FULLMASK, J.hi, jj);
-      labjs[h] = __shfl_sync(FULLMASK, J.lab, jj);
-      x[h] = valid ? Dj[e - sj] : 0;
-      keep[h] = valid && x[h] > loj && x[h] < hij;
-      need[h] = keep[h] && (fjs[h] & 1);
-    }
-    bool f[2] = {false, false};
-    bool bs[2];
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      bs[h] = need[h] && !(fjs[h] & 8);
-      if (need[h] && (fjs[h] & 8)) f[h] = (__ldg((const unsigned*)Pjs[h] + (x[h] >> 5)) >> (x[h] & 31)) & 1u;
-    }
-    if (bs[0] || bs[1]) {
-      bool f0, f1;
-      member2(Pjs[0], bs[0] ? pls[0] : 0, x[0], Pjs[1], bs[1] ? pls[1] : 0, x[1], f0, f1);
-      if (bs[0]) f[0] = f0;
-      if (bs[1]) f[1] = f1;
-    }
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      if (need[h]) keep[h] = (fjs[h] & 4) ? !f[h] : f[h];
-      if (keep[h] && labjs[h] != STM_LAB_ANY) keep[h] = (l2s[glabels[x[h]]] & labjs[h]) != 0;
-      const int eb = e0 + 32 * h;
-      const unsigned km = __ballot_sync(FULLMASK, keep[h]);
-      int a = start - eb, b = incl - eb;
-      a = a < 0 ? 0 : a;
-      b = b > 32 ? 32 : b;
-      unsigned rmask = 0;
-      if (mine && a < b) rmask = (b == 32 ? FULLMASK : ((1u << b) - 1)) & ~((1u << a) - 1);
-      if (count_mode) {
-        jc += __popc(km & rmask);
-      } else {
-        int* Oj = (int*)__shfl_sync(FULLMASK, Oll, j[h]);
-        int base = __shfl_sync(FULLMASK, outc, j[h]);
-        int fl = __shfl_sync(FULLMASK, start, j[h]) - eb;
-        fl = fl < 0 ? 0 : fl;
-        unsigned before = km & ((1u << lane) - 1) & ~((1u << fl) - 1);
-        if (keep[h]) Oj[base + __popc(before)] = x[h];
-        outc += __popc(km & rmask);
-      }
-    }
-  }
-#else
   for (int e0 = 0; e0 < total; e0 += 32) {
     const int e = e0 + lane;
     int j = 0;
@@ -554,7 +421,6 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       if (keep && (fj & 1)) {
         bool f;
         if (fj & 8) f = (__ldg((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
-        else if (STM_WITH_HASH && (fj & 2)) f = ht_has(ht, htmask, x);
         else f = member(Pj, pl, x);
         keep = (fj & 4) ? !f : f;
       }
@@ -564,7 +430,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
     // listing build: injectivity exclusions are applied per element (instead of the
     // count correction below), then every kept element is one embedding
     int uj = 0, cj = 0;
-    if (count_mode) {
+    if (count_mode && !probe) {
       uj = __shfl_sync(FULLMASK, J.u, j);
       cj = __shfl_sync(FULLMASK, J.c, j);
       if (keep && excl)
@@ -582,7 +448,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
     if (count_mode) {
       jc += __popc(km & rmask);
 #if STM_LIST
-      if (km) {
+      if (km && !probe) {
         // PAPER.md:75 Output(C, iter): row = f(0..k-1) in pattern-vertex order, caller's ids
         unsigned long long base = 0;
         if (lane == 0) base = atomicAdd(&w.kp->work->list_n, (unsigned long long)__popc(km));
@@ -610,8 +476,11 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       outc += __popc(km & rmask);
     }
   }
-#endif
   PROF_END(11, total)
+  if (probe) {
+    *outc_lane = (int)jc;
+    return 0;
+  }
   if (!count_mode) {
     if (STM_INSTR && w.kp->count_bytes && mine) w.wbytes += 4ull * (unsigned long long)outc;
     *outc_lane = outc;
@@ -647,25 +516,17 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
 __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un) {
   const StmPlan& P = *w.P;
   Job J;
-  src_slice(w, P.cnt_a, F, u, c, un, J.A, J.alen);
+  if (P.cnt_a.kind != STM_SRC_RAW) node_slice(w, P.cnt_a.idx, F, u, un, J.A, J.alen);
   J.B = nullptr;
   J.blen = 0;
   J.op = P.cnt_op;
   const StmFilter f = P.filt[P.k - 1];
   bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
   J.abm = -1;
-  if (P.cnt_a.kind == STM_SRC_RAW) {
-    const int va = pval(w, P.cnt_a.idx, F, u, c);
-    J.abm = hslot(w, va);
-    narrow_row(w, va, J.A, J.alen, J.lo, J.hi);
-  }
+  if (P.cnt_a.kind == STM_SRC_RAW)
+    row_narrow(w, pval(w, P.cnt_a.idx, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
   J.bbm = -1;
-  if (P.cnt_op != STM_OP_NONE) {
-    const int vb = pval(w, P.cnt_b, F, u, c);
-    row(w, vb, J.B, J.blen);
-    J.bbm = hslot(w, vb);
-    narrow_row(w, vb, J.B, J.blen, J.lo, J.hi);
-  }
+  if (P.cnt_op != STM_OP_NONE) row_narrow(w, pval(w, P.cnt_b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
   J.lab = f.lab;
   J.out = nullptr;
   J.u = u;
@@ -778,22 +639,51 @@ __device__ int node_ub_const(const W& w, int s, int F, int u) {
   }
 }
 
-// Compute the nodes of level F+1 for the m siblings SIB(F+1, 0..m-1); offsets
-// NOFF were assigned by the caller; sizes NSZ are written here.
-__device__ STEP_INL void build_nodes(W& w, int F, int m) {
+// Drop the siblings of frame F+1 whose lane flag `keep` is false (lane t = sibling t < m):
+// the kept siblings move down in order with their slice offsets (and sizes, once built).
+__device__ __forceinline__ int compact_siblings(W& w, int F, int m, bool keep) {
+  const int lane = w.lane;
+  const unsigned km = __ballot_sync(FULLMASK, keep && lane < m);
+  const int nm = __popc(km);
+  if (nm == m) return m;
+  const int dst = __popc(km & ((1u << lane) - 1));
+  const bool mv = (km >> lane) & 1u;
+  const int c = lane < m ? SIB(w, F + 1, lane) : 0;
+  __syncwarp();
+  if (mv) SIB(w, F + 1, dst) = c;
   const StmPlan& P = *w.P;
-  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
-  if (nb == ne) return;
+  for (int s = P.level_begin[F + 1]; s < P.level_begin[F + 2]; ++s) {
+    const int o = lane < m ? NOFF(w, s, lane) : 0, z = lane < m ? NSZ(w, s, lane) : 0;
+    __syncwarp();
+    if (mv) { NOFF(w, s, dst) = o; NSZ(w, s, dst) = z; }
+  }
+  __syncwarp();
+  return nm;
+}
+
+// Compute the nodes of level F+1 for the m siblings SIB(F+1, 0..m-1); offsets
+// NOFF were assigned by the caller; sizes NSZ are written here.  With `prune`
+// (plan.h need / pretest), siblings whose level-(F+1) candidate set cannot supply
+// need[F+1] candidates are dropped first (pre-test on bound-narrowed operands) or
+// after the build; returns the number of siblings kept.
+__device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {
+  const StmPlan& P = *w.P;
+  const int L1 = F + 1;
+  const int nb = P.level_begin[L1], ne = P.level_begin[L1 + 1];
+  if (nb == ne) return m;
   const int u = F >= 1 ? w.h->cur[F] : 0;
   // (reads above are ordered before this write by a full-warp collective)
-  if (w.lane == 0) w.h->lgen[F + 1] += 1;  // level F+1 sets are overwritten: drop stale hashes
-  __syncwarp();
-  for (int st = 0; st < P.n_stages[F + 1]; ++st) {
-    // jobs of this stage: (node, sibling) pairs
+  const bool pre = prune && P.pretest[L1];
+  const StmFilter cf = P.filt[L1];  // the candidate consumer's filter
+  // phase -1: candidate pre-test (probe counts); phases 0..: the level's stages
+  for (int st = pre ? -1 : 0; st < P.n_stages[L1]; ++st) {
+    // jobs of this phase: (node, sibling) pairs
     int nodes_in[STM_MAX_NODES];
     int nn = 0;
-    for (int s = nb; s < ne; ++s)
-      if (P.nodes[s].stage == st) nodes_in[nn++] = s;
+    if (st < 0) nodes_in[nn++] = P.cand[L1].idx;
+    else
+      for (int s = nb; s < ne; ++s)
+        if (P.nodes[s].stage == st) nodes_in[nn++] = s;
     const int njobs_total = nn * m;
     for (int j0 = 0; j0 < njobs_total; j0 += 32) {
       const int jj = j0 + w.lane;
@@ -806,32 +696,52 @@ __device__ STEP_INL void build_nodes(W& w, int F, int m) {
         s = nodes_in[jj / m];
         t = jj % m;
         const StmNode nd = P.nodes[s];
-        const int c = SIB(w, F + 1, t);
+        const int c = SIB(w, L1, t);
         J.c = c;
-        bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
-        if (nd.a_kind == STM_SRC_RAW) {
-          const int va = pval(w, nd.a, F, u, c);
-          row(w, va, J.A, J.alen);
-          J.abm = hslot(w, va);
-          narrow_row(w, va, J.A, J.alen, J.lo, J.hi);
-        } else {
-          node_slice(w, nd.a, F, u, t, J.A, J.alen);
-        }
+        if (st < 0) bounds(w, cf.lo, cf.hi, F, u, c, J.lo, J.hi);  // the consumer's bounds
+        else bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
+        if (nd.a_kind == STM_SRC_RAW) row_narrow(w, pval(w, nd.a, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+        else node_slice(w, nd.a, F, u, t, J.A, J.alen);
         J.a_node = nd.a_kind == STM_SRC_NODE ? P.nodes[nd.a].level + 1 : 0;
-        const int vb = pval(w, nd.b, F, u, c);
-        row(w, vb, J.B, J.blen);
-        J.bbm = hslot(w, vb);
-        narrow_row(w, vb, J.B, J.blen, J.lo, J.hi);
+        row_narrow(w, pval(w, nd.b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
         J.op = nd.op;
-        J.lab = nd.lab;
-        J.out = w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
+        J.lab = st < 0 ? cf.lab : nd.lab;
+        J.out = st < 0 ? nullptr : w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
       }
       int outc = 0;
-      run_jobs(w, J, nj, false, F, 0, &outc);
-      if (w.lane < nj) NSZ(w, s, t) = outc;
-      __syncwarp();
+      run_jobs(w, J, nj, st < 0, F, 0, &outc, st < 0);
+      if (st < 0) {  // pre-test: one job per sibling (nn == 1, m <= 32)
+        m = compact_siblings(w, F, m, outc >= P.need[L1]);
+        if (m == 0) return 0;
+      } else {
+        if (w.lane < nj) NSZ(w, s, t) = outc;
+        __syncwarp();
+      }
     }
   }
+  // post-build check: a candidate node of this level smaller (within the consumer's
+  // bounds) than need[F+1] cannot be extended
+  if (prune && !pre && P.need[L1] > 1 && P.cand[L1].kind == STM_SRC_NODE &&
+      P.nodes[P.cand[L1].idx].level == L1) {
+    bool keep = true;
+    if (w.lane < m) {
+      const int c = SIB(w, L1, w.lane);
+      const int* p;
+      int len;
+      node_slice(w, P.cand[L1].idx, F, u, w.lane, p, len);
+      if (len >= P.need[L1] && (cf.lo | cf.hi)) {
+        int lo, hi;
+        bounds(w, cf.lo, cf.hi, F, u, c, lo, hi);
+        int b = 0, e = len;
+        if (lo >= 0) b = lbound(p, len, lo + 1);
+        if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
+        len = e - b;
+      }
+      keep = len >= P.need[L1];
+    }
+    m = compact_siblings(w, F, m, keep);
+  }
+  return m;
 }
 
 // ----------------------------------------------------------------------------
@@ -1080,17 +990,19 @@ __device__ STEP_INL void fused_count(W& w, int F) {
 // ----------------------------------------------------------------------------
 // work acquisition: root chunks, local steal, global steal (Sec. V)
 // ----------------------------------------------------------------------------
-__device__ __noinline__ bool try_chunk(W& w) {
-  const StmKParams& kp = *w.kp;
-  int b = -1, e = -1;
+__device__ __noinline__ bool try_chunk(const StmKParams& kp) {
+  W w = make_w(kp);
+  int b = -1, e = -1, from = -1;
   if (w.lane == 0) {
+    unsigned ex = w.h->exhausted;
     for (int i = 0; i < kp.world && b < 0; ++i) {
       int r = (kp.rank + i) % kp.world;
-      if (!kp.cursors[r] || (w.exhausted & (1u << r))) continue;
+      if (!kp.cursors[r] || (ex & (1u << r))) continue;
       unsigned long long idx = atomicAdd(kp.cursors[r], 1ull);
       long long c = (long long)r + (long long)kp.world * (long long)idx;
       long long rb = kp.root_lo + c * (long long)kp.chunk;
       if (rb < kp.n) {
+        from = r;
         b = (int)rb;
         e = (int)min((long long)kp.n, rb + kp.chunk);
         if (kp.root_desc) {  // chunk c covers [lo + n - e, lo + n - b): the highest ids first
@@ -1099,16 +1011,16 @@ __device__ __noinline__ bool try_chunk(W& w) {
           b = nb;
         }
       } else {
-        w.exhausted |= 1u << r;
+        ex |= 1u << r;
       }
     }
+    w.h->exhausted = ex;
+#if STM_PROFILE
+    if (b < 0 && w.h->first_dry == 0) w.h->first_dry = clock64();
+#endif
   }
   b = bcast(b);
   e = bcast(e);
-  w.exhausted = __shfl_sync(FULLMASK, w.exhausted, 0);
-#if STM_PROFILE
-  if (b < 0 && w.first_dry == 0) w.first_dry = clock64();
-#endif
   if (b < 0) return false;
   lock_ws(w, w.h);
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
@@ -1118,7 +1030,10 @@ __device__ __noinline__ bool try_chunk(W& w) {
     w.h->L = 0;
   }
   unlock_ws(w, w.h);
-  if (w.lane == 0) atomicAdd(&kp.work->n_chunks, 1ull);
+  if (w.lane == 0) {
+    atomicAdd(&kp.work->n_chunks, 1ull);
+    if (from != kp.rank) atomicAdd(&kp.work->n_peer_chunks, 1ull);
+  }
   return true;
 }
 
@@ -1133,12 +1048,11 @@ struct SplitPick {
   int F, kind, t;
 };
 
-__device__ __forceinline__ SplitPick pick_split(const W& w, volatile WarpHdr* v) {
+__device__ __forceinline__ SplitPick pick_split(int stop, volatile WarpHdr* v) {
   const int L = v->L;
   const int r = v->root_end - v->root_it;
   const int t = (L > 0) ? (r + 1) / 2 : r / 2;
   if (t >= 1) return {0, 0, t};
-  const int stop = w.kp->stop_level;
   for (int F = 1; F <= L && F < stop; ++F) {
     const int cur = v->cur[F], nsib = v->nsib[F];
     if (cur >= nsib) continue;
@@ -1156,8 +1070,9 @@ __device__ __forceinline__ SplitPick pick_split(const W& w, volatile WarpHdr* v)
 }
 
 // Split the stack of `v` (caller holds v's lock).  Returns false if nothing.
-__device__ __noinline__ bool split_stack(const W& w, volatile WarpHdr* v, volatile int* vsib, StmTask& T) {
-  const SplitPick s = pick_split(w, v);
+__device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr* v, volatile int* vsib,
+                                        StmTask& T) {
+  const SplitPick s = pick_split(kp.stop_level, v);
   if (s.F < 0) return false;
   if (s.kind == 0) {
     T.level = 0;
@@ -1183,34 +1098,46 @@ __device__ __noinline__ bool split_stack(const W& w, volatile WarpHdr* v, volati
 
 // amount-of-work score of a stack (higher = better victim; 0 = nothing a split
 // would take), racy read without the lock
-__device__ __forceinline__ int steal_score(const W& w, volatile WarpHdr* v) {
-  const SplitPick s = pick_split(w, v);
+__device__ __forceinline__ int steal_score(int stop, volatile WarpHdr* v) {
+  const SplitPick s = pick_split(stop, v);
   if (s.F < 0) return 0;
   if (s.F == 0) return 1 << 30;
   return ((STM_KMAX - s.F) << 24) + min(s.t * (s.kind == 1 ? 1024 : 1), (1 << 24) - 1);
 }
 
-__device__ volatile WarpHdr* warp_hdr(const W& w, int wid);
 
-// debug watchdog: true (and a state dump) once the launch has run too long
-__device__ __noinline__ bool watchdog(const W& w, long long t0, const char* where) {
-  if (!w.kp->watchdog_cycles || clock64() - t0 < w.kp->watchdog_cycles) return false;
+__device__ __forceinline__ long long gtimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Failure detection (stm_tuning.watchdog_ms): true once the launch has run longer
+// than watchdog_ns of wall time; the launch then aborts and reports STM_ETIMEOUT
+// (work->overflow = 2), never a partial count.  STM_DEBUG builds also dump state.
+__device__ __noinline__ bool watchdog(const StmKParams& kp, long long t0, const char* where) {
+  if (!kp.watchdog_ns || gtimer() - t0 < kp.watchdog_ns) return false;
+  W w = make_w(kp);
   if (w.lane == 0) {
-    int first = atomicExch(&w.kp->work->overflow, 2);
+    atomicExch(&w.kp->work->overflow, 2);
+#if STM_DEBUG
     volatile WarpHdr* h = w.h;
-    printf("WATCHDOG %s blk %d warp %d L=%d root=[%d,%d) nsib1=%d cur1=%d it1=%d end1=%d idle_blocks=%d mask=%x leader=%d is_idle=%d mail=%d first=%d\n",
+    printf("WATCHDOG %s blk %d warp %d L=%d root=[%d,%d) nsib1=%d cur1=%d it1=%d end1=%d idle_blocks=%d mask=%x leader=%d is_idle=%d mail=%d\n",
            where, blockIdx.x, w.wid, h->L, h->root_it, h->root_end, h->nsib[1], h->cur[1], h->it[1], h->end[1],
            *(volatile int*)&w.kp->work->idle_blocks, w.bh->idle_mask, w.bh->leader,
-           w.kp->slots[blockIdx.x].is_idle, w.kp->slots[blockIdx.x].mail_full, first);
+           w.kp->slots[blockIdx.x].is_idle, w.kp->slots[blockIdx.x].mail_full);
+#else
+    (void)where;
+#endif
   }
   __syncwarp();
   return true;
 }
-__device__ volatile int* warp_sib(const W& w, int wid);
 
 // Rebuild this warp's stack from a task (the receiver recomputes the sets of
 // levels 1..T.level from the prefix).
-__device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
+__device__ __noinline__ void adopt_task(const StmKParams& kp, const StmTask& T) {
+  W w = make_w(kp);
   const int k = w.P->k;
   if (T.level == 0) {
     lock_ws(w, w.h);
@@ -1238,7 +1165,7 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
       if (w.lane == 0)
         for (int s = P.level_begin[i]; s < P.level_begin[i + 1]; ++s) NOFF(w, s, 0) = 0;
       __syncwarp();
-      build_nodes(w, i - 1, 1);
+      build_nodes(w, i - 1, 1, false);  // a stolen prefix is rebuilt as given
     }
     int len = src_len(w, i, 0);
     HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
@@ -1253,14 +1180,24 @@ __device__ __noinline__ void adopt_task(W& w, const StmTask& T) {
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->L = l;
   unlock_ws(w, w.h);
+  flush_instr(w);  // the rebuild's set operations count toward W
 }
 
-__device__ __noinline__ bool try_local_steal(W& w) {
-  const int nw = w.kp->block_warps;
+__device__ __forceinline__ volatile WarpHdr* warp_hdr(const W& w, int wid) {
+  const int wb = warp_bytes(w.P->k, w.P->n_nodes, w.kp->ht_slots);
+  return (volatile WarpHdr*)(stm_smem + sizeof(BlockHdr) + (size_t)wid * wb);
+}
+__device__ __forceinline__ volatile int* warp_sib(const W& w, int wid) {
+  return (volatile int*)((volatile unsigned char*)warp_hdr(w, wid) + sizeof(WarpHdr));
+}
+
+__device__ __noinline__ bool try_local_steal(const StmKParams& kp) {
+  W w = make_w(kp);
+  const int nw = kp.block_warps;
   // pick the best victim (racy scores), then split under its lock
   int best = -1, bs = 0;
   if (w.lane < nw && w.lane != w.wid) {
-    int s = steal_score(w, warp_hdr(w, w.lane));
+    int s = steal_score(kp.stop_level, warp_hdr(w, w.lane));
     if (s > 0) { best = w.lane; bs = s; }
   }
   // warp argmax (lowest id on ties)
@@ -1275,7 +1212,7 @@ __device__ __noinline__ bool try_local_steal(W& w) {
   StmTask T;
   int ok = 0;
   lock_ws(w, v);
-  if (w.lane == 0) ok = split_stack(w, v, warp_sib(w, best), T);
+  if (w.lane == 0) ok = split_stack(kp, v, warp_sib(w, best), T);
   unlock_ws(w, v);
   ok = bcast(ok);
   if (!ok) return false;
@@ -1283,25 +1220,28 @@ __device__ __noinline__ bool try_local_steal(W& w) {
   T.b = bcast(T.b);
   T.e = bcast(T.e);
   for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
-  if (w.lane == 0) atomicAdd(&w.kp->work->n_local_steals, 1ull);
-  adopt_task(w, T);
+  if (w.lane == 0) atomicAdd(&kp.work->n_local_steals, 1ull);
+  adopt_task(kp, T);
   return true;
 }
 
 // donor side of Fig. 6: give half of my shallowest work to an idle block
-__device__ __noinline__ void maybe_donate(W& w) {
-  const StmKParams& kp = *w.kp;
-  // the idle-block count lives in L2: look at it on every 8th opportunity only
-  if ((++w.donate_tick & (unsigned)w.kp->donate_mask) != 0) return;
+__device__ __noinline__ void maybe_donate(const StmKParams& kp) {
+  W w = make_w(kp);
+  // the idle-block count lives in L2: look at it on every (donate_mask+1)-th opportunity
+  unsigned tick = 0;
+  if (w.lane == 0) tick = ++w.h->donate_tick;
+  tick = __shfl_sync(FULLMASK, tick, 0);
+  if ((tick & (unsigned)kp.donate_mask) != 0) return;
   int idle = 0;
   if (w.lane == 0) idle = *(volatile int*)&kp.work->idle_blocks;
   idle = bcast(idle);
   if (idle <= 0) return;
   // only donate what a split can actually take
-  if (pick_split(w, w.h).F < 0) return;
+  if (pick_split(kp.stop_level, w.h).F < 0) return;
   const int nb = gridDim.x;
   int target = -1;
-  const int off = (int)((blockIdx.x * 37u + w.wid * 11u + w.donate_tick) % (unsigned)nb);
+  const int off = (int)((blockIdx.x * 37u + w.wid * 11u + tick) % (unsigned)nb);
   for (int b0 = 0; b0 < min(nb, 64) && target < 0; b0 += 32) {
     int b = (off + b0 + w.lane) % nb;
     bool cand = (b0 + w.lane < nb) && b != (int)blockIdx.x &&
@@ -1320,7 +1260,7 @@ __device__ __noinline__ void maybe_donate(W& w) {
   StmTask T;
   int ok = 0;
   lock_ws(w, w.h);
-  if (w.lane == 0) ok = split_stack(w, w.h, w.sib, T);
+  if (w.lane == 0) ok = split_stack(kp, w.h, w.sib, T);
   unlock_ws(w, w.h);
   if (w.lane == 0) {
     if (!ok) {
@@ -1342,11 +1282,11 @@ __device__ __noinline__ void maybe_donate(W& w) {
 }
 
 // No more local work: returns true with new work adopted, false on termination.
-__device__ __noinline__ bool acquire_work(W& w, long long t0) {
-  const StmKParams& kp = *w.kp;
-  if (try_chunk(w)) return true;
+__device__ __noinline__ bool acquire_work(const StmKParams& kp, long long t0) {
+  W w = make_w(kp);
+  if (try_chunk(kp)) return true;
   if (!kp.local_steal && !kp.global_steal) return false;
-  if (kp.local_steal && try_local_steal(w)) return true;
+  if (kp.local_steal && try_local_steal(kp)) return true;
   BlockHdr* bh = w.bh;
   const unsigned all = (kp.block_warps == 32) ? FULLMASK : ((1u << kp.block_warps) - 1);
   const unsigned me = 1u << w.wid;
@@ -1360,7 +1300,7 @@ __device__ __noinline__ bool acquire_work(W& w, long long t0) {
     (void)bcast(got);
   }
   for (int spin = 0;; ++spin) {
-    if ((spin & 1023) == 1023 && watchdog(w, t0, "acquire")) return false;
+    if ((spin & 1023) == 1023 && watchdog(kp, t0, "acquire")) return false;
     int done = 0, leader = -1;
     if (w.lane == 0) {
       done = *(volatile int*)&bh->done;
@@ -1413,7 +1353,7 @@ __device__ __noinline__ bool acquire_work(W& w, long long t0) {
         T.b = bcast(T.b);
         T.e = bcast(T.e);
         for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
-        adopt_task(w, T);
+        adopt_task(kp, T);
         return true;
       }
       if (nidle >= (int)gridDim.x) {
@@ -1426,8 +1366,11 @@ __device__ __noinline__ bool acquire_work(W& w, long long t0) {
       // while a stolen task is in flight
       if (w.lane == 0) atomicAnd(&bh->idle_mask, (int)~me);
       __syncwarp();
-      if (try_local_steal(w)) { w.steal_fails = 0; return true; }
-      w.steal_fails = min(w.steal_fails + 1, w.kp->backoff_max);
+      if (try_local_steal(kp)) {
+        if (w.lane == 0) w.h->steal_fails = 0;
+        return true;
+      }
+      if (w.lane == 0) w.h->steal_fails = min(w.h->steal_fails + 1, kp.backoff_max);
       if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
       old = bcast(old);
       if ((((unsigned)old) | me) == all) {
@@ -1435,18 +1378,9 @@ __device__ __noinline__ bool acquire_work(W& w, long long t0) {
         __syncwarp();
       }
     }
-    if (w.lane == 0) __nanosleep(32u << w.steal_fails);  // back off while nothing can be stolen
+    if (w.lane == 0) __nanosleep(32u << w.h->steal_fails);  // back off while nothing can be stolen
     __syncwarp();
   }
-}
-
-__device__ volatile WarpHdr* warp_hdr(const W& w, int wid) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  int wb = warp_bytes(w.P->k, w.P->n_nodes, w.kp->ht_slots);
-  return (volatile WarpHdr*)(smem + sizeof(BlockHdr) + (size_t)wid * wb);
-}
-__device__ volatile int* warp_sib(const W& w, int wid) {
-  return (volatile int*)((volatile unsigned char*)warp_hdr(w, wid) + sizeof(WarpHdr));
 }
 
 }  // namespace
@@ -1455,52 +1389,25 @@ __device__ volatile int* warp_sib(const W& w, int wid) {
 // the kernel
 // ----------------------------------------------------------------------------
 __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
-  extern __shared__ __align__(16) unsigned char smem[];
   const StmPlan& P = kp.plan;
-  BlockHdr* bh = (BlockHdr*)smem;
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  BlockHdr* bh = (BlockHdr*)stm_smem;
+  const int lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     bh->idle_mask = 0;
     bh->leader = -1;
     bh->done = 0;
   }
   for (int i = threadIdx.x; i < 256; i += blockDim.x) bh->lab2slot[i] = kp.lab2slot[i];
-  const int wb = warp_bytes(P.k, P.n_nodes, kp.ht_slots);
-  unsigned char* wbase = smem + sizeof(BlockHdr) + (size_t)wid * wb;
-  W w;
-  w.kp = &kp;
-  w.P = &P;
-  w.h = (volatile WarpHdr*)wbase;
-  w.sib = (volatile int*)(wbase + sizeof(WarpHdr));
-  w.noff = (int*)(wbase + sizeof(WarpHdr) + P.k * STM_RMAX * 4);
-  w.nsz = w.noff + P.n_nodes * STM_UMAX;
-  w.ht = w.nsz + P.n_nodes * STM_UMAX;
-  w.ht_mask = 0;
-  w.ht_ptr = 0;
-  w.ht_len = -1;
-  w.ht_gen = 0;
-  w.bh = bh;
-  const long long gw = (long long)blockIdx.x * kp.block_warps + wid;
-  w.arena = kp.arena + (size_t)gw * (size_t)P.n_nodes * (size_t)kp.cap;
-  w.lane = lane;
-  w.wid = wid;
-  w.exhausted = 0;
-  w.cnt = 0;
-  w.gather_calls = 0;
-  w.donate_tick = 0;
-  w.steal_fails = 0;
-  w.wbytes = w.wmerge = w.wjobs = 0;
-  w.idle_cyc = 0;
-#if STM_PROFILE
-  for (int i = 0; i < STM_PROF_N; ++i) w.prof_cyc[i] = w.prof_cnt[i] = w.prof_items[i] = 0;
-  w.first_dry = 0;
-#endif
+  W w = make_w(kp);
   if (lane == 0) {
     w.h->lock = 0;
     w.h->L = 0;
     w.h->root_it = 0;
     w.h->root_end = 0;
-    for (int i = 0; i <= STM_KMAX; ++i) w.h->lgen[i] = 1;
+    w.h->exhausted = 0;
+    w.h->donate_tick = 0;
+    w.h->steal_fails = 0;
+    w.h->first_dry = 0;
     for (int i = 0; i < STM_KMAX; ++i) {
       w.h->nsib[i] = 0;
       w.h->cur[i] = 0;
@@ -1514,9 +1421,10 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
   const int U = max(1, min(kp.unroll, STM_UMAX));
   const bool fused = P.count_mode == STM_COUNT_FUSED;
   const long long t0 = clock64();
+  const long long wd0 = gtimer();
   unsigned iter = 0;
   for (;;) {
-    if ((++iter & 255) == 0 && watchdog(w, t0, "main")) break;
+    if ((++iter & 255) == 0 && watchdog(kp, wd0, "main")) break;
     int L = w.h->L;
     if (L == 0) {
       const bool lk = stealing(w);
@@ -1549,7 +1457,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
         // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
         const long long ta = (STM_INSTR && kp.count_bytes) ? clock64() : 0;
         PROF_BEGIN(7)
-        const bool got = acquire_work(w, t0);
+        const bool got = acquire_work(kp, wd0);
         PROF_END(7, got)
         if (STM_INSTR && kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
         if (!got) break;
@@ -1572,7 +1480,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     const bool lk = locked_frame(w, F);
     if (kp.global_steal && F < kp.detect_level && F < kp.stop_level) {
       PROF_BEGIN(6)
-      maybe_donate(w);
+      maybe_donate(kp);
       PROF_END(6, 0)
     }
     if (lk) lock_ws(w, w.h);
@@ -1608,8 +1516,9 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     if (lk) unlock_ws(w, w.h);
     // build frame F+1 from the batch
     PROF_BEGIN(3)
-    build_nodes(w, F, m);
+    m = build_nodes(w, F, m, true);
     PROF_END(3, m)
+    if (m == 0) continue;  // every sibling of the batch was pruned: gather the next one
     if (F + 1 == k - 1) {  // frame-count mode
       PROF_BEGIN(4)
       frame_count(w, m);
@@ -1641,23 +1550,34 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     atomicAdd(&kp.work->prof[3 * STM_PROF_N], (unsigned long long)(now - t0));
     // tail shape (clock64 is per SM; SMs start within a few us of each other)
     atomicMax(&kp.work->prof[3 * STM_PROF_N + 1], (unsigned long long)(now - t0));
-    atomicAdd(&kp.work->prof[3 * STM_PROF_N + 2], (unsigned long long)(w.first_dry ? w.first_dry - t0 : now - t0));
-    atomicMax(&kp.work->prof[3 * STM_PROF_N + 3], (unsigned long long)(w.first_dry ? w.first_dry - t0 : now - t0));
+    const long long fd = w.h->first_dry;
+    atomicAdd(&kp.work->prof[3 * STM_PROF_N + 2], (unsigned long long)(fd ? fd - t0 : now - t0));
+    atomicMax(&kp.work->prof[3 * STM_PROF_N + 3], (unsigned long long)(fd ? fd - t0 : now - t0));
   }
 #endif
   if (STM_INSTR && kp.count_bytes) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      w.wbytes += __shfl_xor_sync(FULLMASK, w.wbytes, o);
-      w.wmerge += __shfl_xor_sync(FULLMASK, w.wmerge, o);
-      w.wjobs += __shfl_xor_sync(FULLMASK, w.wjobs, o);
-    }
+    flush_instr(w);
     if (lane == 0) {
       atomicAdd(&kp.work->idle_cycles, w.idle_cyc);
       atomicAdd(&kp.work->warp_cycles, (unsigned long long)(clock64() - t0));
-      atomicAdd(&kp.work->alg_bytes, w.wbytes);
-      atomicAdd(&kp.work->merge_bytes, w.wmerge);
-      atomicAdd(&kp.work->n_jobs, w.wjobs);
+    }
+  }
+  // The last block to finish publishes the async result record (stm_async_result):
+  // every warp's count is ordered before its block's arrival by the fence.
+  if (kp.result) {
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      const unsigned done = atomicAdd(&kp.work->blocks_done, 1u);
+      if (done == gridDim.x - 1) {
+        __threadfence();
+        volatile StmWork* vw = kp.work;
+        const int ov = vw->overflow;
+        kp.result[0] = ov ? 0ull : vw->count;
+        kp.result[1] = ov == 2 ? 6ull /* STM_ETIMEOUT */ : ov ? 5ull /* STM_EOVERFLOW */ : 0ull;
+        kp.result[2] = vw->n_chunks;
+        kp.result[3] = vw->n_peer_chunks;
+      }
     }
   }
 }
@@ -1677,15 +1597,16 @@ static const void* STM_SYM(kernel_fn)(int variant) {
 }
 
 #if !STM_INSTR && !STM_LIST
-int stm_drive_compiled() { return STM_DRIVE_RATIO; }
-int stm_hash_compiled() { return STM_WITH_HASH; }
+int stm_drive_compiled() { return 0; }  // drive_ratio / hash sets: measured slower, removed
+int stm_hash_compiled() { return 0; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
   return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);
 }
 #endif
 
-int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm) {
+int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                           int* blocks_per_sm) {
   const void* fn = STM_SYM(kernel_fn)(variant);
   int smem = stm_smem_bytes(block_warps, k, n_nodes, ht_slots);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -1703,7 +1624,7 @@ int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int
   const double need = (double)want * (smem + 1024);
   int pct = (int)std::ceil(100.0 * need / (228.0 * 1024.0));
   pct = std::max(0, std::min(100, pct));
-  if (const char* cv = getenv("STM_CARVEOUT")) pct = atoi(cv);  // experiments: -1 = leave the driver default
+  if (carveout != 0) pct = carveout;  // stm_tuning.carveout_pct: -1 = leave the driver default
   if (pct >= 0) {
     e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
     if (e != cudaSuccess) return (int)e;

@@ -3,6 +3,8 @@
 #pragma once
 #include <stdint.h>
 
+#include <cuda_runtime.h>  // int4
+
 #include "plan.h"
 
 // A unit of stealable work (Sec. V).  level 0: root-ID range
@@ -27,8 +29,11 @@ struct StmTask {
 struct StmWork {
   unsigned long long count;       // result accumulator (mod 2^64)
   int32_t idle_blocks;            // blocks registered idle (Fig. 6 is_idle count)
-  int32_t overflow;               // set if any capacity check fails
+  int32_t overflow;               // 1: a capacity check failed, 2: the watchdog expired (no count)
   unsigned long long n_local_steals, n_global_steals, n_chunks;
+  unsigned long long n_peer_chunks;  // chunks taken from peer ranks' cursors
+  unsigned int blocks_done;          // blocks that finished (the last one writes the async result)
+  unsigned int pad0;
   unsigned long long alg_bytes;    // SURVEY.md 8(d) W = sum W_op (instrumented launches only)
   unsigned long long merge_bytes;  // W_merge = sum 4(|A|+|B|)
   unsigned long long n_jobs;
@@ -48,14 +53,13 @@ struct StmBlockSlot {             // per block, global memory (Fig. 6)
 
 struct StmKParams {
   StmPlan plan;
-  const int64_t* row_ptr;
+  const int4* vrec;               // [n] packed (row start, degree, out_start, hub slot), kernel.cu vrec()
   const int32_t* col_idx;
   const uint8_t* labels;          // dense graph label ids, or NULL
-  // Hub adjacency bitmaps: hub_slot[v] >= 0 selects the
+  // Hub adjacency bitmaps: vrec[v].w >= 0 selects the
   // n-bit row bitmaps[slot * bm_words ...] of N(v); membership probes into such a
-  // row read one word instead of a binary search.  hub_slot == NULL: none.
-  const int32_t* out_start;       // [n]: index in N(v) of the first neighbour > v (NULL: none)
-  const int32_t* hub_slot;
+  // row read one word instead of a binary search.
+  int32_t split;                  // 1: narrow rows with the out_start split of vrec (stm_tuning.narrow_split 0)
   const uint32_t* bitmaps;
   int64_t bm_words;
   int64_t n;                      // root space end: roots are [root_lo, n)
@@ -78,7 +82,8 @@ struct StmKParams {
   int32_t donate_mask;            // donors look for idle blocks every (mask+1)-th opportunity
   int32_t drive_ratio;            // drive B while |B| <= drive_ratio |A| when A is shared by all jobs (0/1 = shorter)
   int32_t backoff_max;            // idle warps sleep up to 32 << backoff_max ns between steal attempts
-  long long watchdog_cycles;      // debug: abort (set work->overflow = 2) after this many cycles; 0 = off
+  long long watchdog_ns;          // abort (work->overflow = 2) after this much %globaltimer time; 0 = off
+  unsigned long long* result;     // stm_async_result {count, status, chunks, peer_chunks} or NULL
   const void* l2_window_base;     // L2 persisting access-policy window (0 bytes = none)
   long long l2_window_bytes;
   uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
@@ -96,6 +101,9 @@ int stm_launch(int variant, const StmKParams& kp, int grid, void* stream);
 int stm_launch_instr(int variant, const StmKParams& kp, int grid, void* stream);  // instrumented build
 int stm_launch_list(int variant, const StmKParams& kp, int grid, void* stream);   // listing build
 // max co-resident blocks per SM for the given block size
-int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
-int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
-int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_slots, int* blocks_per_sm);
+// carveout: stm_tuning.carveout_pct (0 = auto, -1 = driver default, else percent)
+int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout, int* blocks_per_sm);
+int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                        int* blocks_per_sm);
+int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                       int* blocks_per_sm);

@@ -116,8 +116,14 @@ extern "C" stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags
   if (!g) return stm_fail(STM_EINVAL, "graph is NULL");
   if (k < 2 || k > kMotifKMax) return stm_fail(STM_EUNSUPPORTED, "motif size k=%d outside 2..%d", k, kMotifKMax);
   if (!n_motifs || !counts) return stm_fail(STM_EINVAL, "NULL output");
-  if (flags & ~(uint32_t)(STM_VERTEX_INDUCED | STM_NO_CODE_MOTION | STM_LAZY_UNBOUNDED))
-    return stm_fail(STM_EINVAL, "census flags: only STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_LAZY_UNBOUNDED");
+  if (flags & ~(uint32_t)(STM_VERTEX_INDUCED | STM_NO_CODE_MOTION | STM_LAZY_UNBOUNDED | STM_AUTO_ORDER))
+    return stm_fail(STM_EINVAL,
+                    "census flags: only STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_LAZY_UNBOUNDED, STM_AUTO_ORDER");
+  // cost-based orders by default: the caller's statistics, else the graph's own (computed
+  // at load); STM_AUTO_ORDER keeps the compiler's greedy order
+  stm_graph_stats gstats;
+  if (!stats && !(flags & STM_AUTO_ORDER) && stm_graph_get_stats(g, &gstats) == STM_OK) stats = &gstats;
+  flags &= ~(uint32_t)STM_AUTO_ORDER;
   const auto& cat = catalog(k);
   if (capacity < (int)cat.size())
     return stm_fail(STM_EINVAL, "capacity %d < %zu motifs of size %d", capacity, cat.size(), k);

@@ -75,4 +75,13 @@ struct StmPlan {
   int8_t cnt_b;                      // position, or -1 when op == STM_OP_NONE
   int8_t cnt_op;
   int8_t pad[2];
+  // Candidate-set pruning: need[l] = the minimal size of level l's
+  // candidate set (within its bounds) for any embedding to extend the prefix -- v_l itself
+  // plus every later v_m that must also come from it; a sibling whose level-(l) set is
+  // smaller is dropped before its frame is entered.  pretest[l] = 1: level l's candidate
+  // source is an unbounded stage-0 node of level l with a bounded consumer -- its size
+  // within the consumer's bounds is counted on bound-narrowed operands first, and the
+  // level's sets are materialised only for the siblings that pass.
+  int8_t need[STM_KMAX];
+  int8_t pretest[STM_KMAX];
 };

@@ -6,6 +6,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <tuple>
 #include <mutex>
 #include <new>
 #include <thread>
@@ -91,17 +92,22 @@ struct stm_graph {
   // it could not be built; then the kernel narrows by binary search alone)
   int32_t* d_out_start = nullptr;
   int32_t* d_rout_start = nullptr;
-  // Hub adjacency bitmaps, per numbering ([0] caller's ids, [1] degree-ranked),
-  // built lazily by the first launch that asks for them.
+  // Hub adjacency bitmaps per (numbering, min degree, budget), built lazily by the
+  // first launch that asks for them and kept until the
+  // graph is freed: a launch on another stream may still read a set another call no
+  // longer wants, so no set is ever freed or rebuilt while the graph is alive.
   struct HubBitmaps {
     int32_t* slot = nullptr;   // [n]: bitmap slot of v, -1 = none
     uint32_t* bits = nullptr;  // [n_hubs][words]
     int64_t words = 0, n_hubs = 0;
-    int min_deg = -2;          // parameters the cached copy was built with (-2 = never built)
-    int64_t budget = -1;
-  } hub[2];
+    int4* vrec = nullptr;      // [n] packed (row start, degree, out_start, hub slot) for this set
+  };
+  std::map<std::tuple<int, int, int64_t>, HubBitmaps> hubs;  // (ranked, min_deg, budget) -> set
   std::mutex mu;
   std::map<void*, Scratch> scratch;  // per stream
+  // degree / label statistics of the graph (NEXT-2 cost model), computed at load
+  bool has_stats = false;
+  stm_graph_stats stats;
 };
 
 // ---------------------------------------------------------------------------- load
@@ -272,56 +278,84 @@ __global__ void hub_fill(int64_t n, int64_t H, const int32_t* rank2orig, const i
 static void free_hub(stm_graph::HubBitmaps& h) {
   cudaFree(h.slot);
   cudaFree(h.bits);
+  cudaFree(h.vrec);
   h = stm_graph::HubBitmaps();
 }
 
-// Makes g->hub[ranked] hold bitmaps of every vertex with degree >= min_deg, at most
-// budget bytes (highest degrees first).  Speed only: on any failure there are none.
-static const stm_graph::HubBitmaps* ensure_hub(stm_graph* g, bool ranked, int min_deg, int64_t budget) {
-  stm_graph::HubBitmaps& h = g->hub[ranked ? 1 : 0];
-  if (min_deg < 0 || !g->ranked || g->n < 1) return nullptr;
-  if (h.min_deg == min_deg && h.budget == budget) return h.n_hubs ? &h : nullptr;
-  free_hub(h);
-  h.min_deg = min_deg;
-  h.budget = budget;
-  const int64_t n = g->n;
-  const int64_t words = (n + 31) / 32;
-  const int64_t hmax = budget / (words * 4);
-  unsigned long long* d = nullptr;
-  unsigned long long H = 0;
-  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 4096);
-  cudaError_t e = cudaMalloc(&d, sizeof H);
-  if (e == cudaSuccess) e = cudaMemset(d, 0, sizeof H);
-  if (e == cudaSuccess) count_deg_ge<<<grid, 256>>>(g->d_rrow_ptr, n, std::max(min_deg, 1), d);
-  if (e == cudaSuccess) e = cudaMemcpy(&H, d, sizeof H, cudaMemcpyDeviceToHost);
-  cudaFree(d);
-  H = std::min<unsigned long long>(H, (unsigned long long)std::max<int64_t>(hmax, 0));
-  if (e != cudaSuccess || H == 0) {
-    cudaGetLastError();
-    return nullptr;
+// packed per-vertex records of one numbering and hub set (kernel.cu vrec())
+__global__ void vrec_fill(const int64_t* rp, int64_t n, const int32_t* out_start, const int32_t* slot, int4* out) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = rp[v];
+    out[v] = make_int4((int)(uint32_t)b, (int)(rp[v + 1] - b), out_start ? out_start[v] : -1, slot ? slot[v] : -1);
   }
-  e = cudaMalloc(&h.slot, sizeof(int32_t) * n);
-  if (e == cudaSuccess) e = cudaMalloc(&h.bits, sizeof(uint32_t) * (size_t)words * H);
-  if (e == cudaSuccess) e = cudaMemset(h.slot, 0xFF, sizeof(int32_t) * n);
-  if (e == cudaSuccess) e = cudaMemset(h.bits, 0, sizeof(uint32_t) * (size_t)words * H);
-  if (e == cudaSuccess) {
-    const int32_t* r2o = ranked ? nullptr : g->d_rank2orig;
-    hub_slots<<<(unsigned)std::min<unsigned long long>((H + 255) / 256, 4096), 256>>>(n, (int64_t)H, r2o, h.slot);
-    hub_fill<<<(unsigned)std::min<unsigned long long>(H, 65535), 256>>>(
-        n, (int64_t)H, r2o, ranked ? g->d_rrow_ptr : g->d_row_ptr, ranked ? g->d_rcol_idx : g->d_col_idx, words,
-        h.bits);
+}
+
+// The launch-side view of a graph for one numbering (`ranked`) and hub set: hub
+// bitmaps of every vertex with degree >= min_deg (at most budget bytes, highest
+// degrees first; min_deg < 0: none) and the packed vertex records that point into
+// them.  Caller holds g->mu.  Built once per key and kept until the graph is freed.
+// Returns NULL only if the records cannot be built (the bitmaps are speed only: on
+// failure the set simply has none).
+static const stm_graph::HubBitmaps* ensure_hub(stm_graph* g, bool ranked, int min_deg, int64_t budget) {
+  if (min_deg < 0 || !g->ranked) { min_deg = -1; budget = 0; }
+  const auto key = std::make_tuple(ranked ? 1 : 0, min_deg, budget);
+  auto it = g->hubs.find(key);
+  if (it != g->hubs.end()) return it->second.vrec ? &it->second : nullptr;
+  stm_graph::HubBitmaps& h = g->hubs[key];
+  const int64_t n = g->n;
+  const int64_t* rp = ranked ? g->d_rrow_ptr : g->d_row_ptr;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 4096);
+  cudaError_t e = cudaSuccess;
+  if (min_deg >= 0 && n > 0) {
+    const int64_t words = (n + 31) / 32;
+    const int64_t hmax = budget / (words * 4);
+    unsigned long long* d = nullptr;
+    unsigned long long H = 0;
+    e = cudaMalloc(&d, sizeof H);
+    if (e == cudaSuccess) e = cudaMemset(d, 0, sizeof H);
+    if (e == cudaSuccess) count_deg_ge<<<grid, 256>>>(g->d_rrow_ptr, n, std::max(min_deg, 1), d);
+    if (e == cudaSuccess) e = cudaMemcpy(&H, d, sizeof H, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    H = std::min<unsigned long long>(H, (unsigned long long)std::max<int64_t>(hmax, 0));
+    if (e == cudaSuccess && H > 0) {
+      e = cudaMalloc(&h.slot, sizeof(int32_t) * n);
+      if (e == cudaSuccess) e = cudaMalloc(&h.bits, sizeof(uint32_t) * (size_t)words * H);
+      if (e == cudaSuccess) e = cudaMemset(h.slot, 0xFF, sizeof(int32_t) * n);
+      if (e == cudaSuccess) e = cudaMemset(h.bits, 0, sizeof(uint32_t) * (size_t)words * H);
+      if (e == cudaSuccess) {
+        const int32_t* r2o = ranked ? nullptr : g->d_rank2orig;
+        hub_slots<<<(unsigned)std::min<unsigned long long>((H + 255) / 256, 4096), 256>>>(n, (int64_t)H, r2o, h.slot);
+        hub_fill<<<(unsigned)std::min<unsigned long long>(H, 65535), 256>>>(
+            n, (int64_t)H, r2o, rp, ranked ? g->d_rcol_idx : g->d_col_idx, words, h.bits);
+        e = cudaGetLastError();
+        if (e == cudaSuccess) e = cudaDeviceSynchronize();
+      }
+      if (e == cudaSuccess) {
+        h.words = words;
+        h.n_hubs = (int64_t)H;
+      }
+    }
+    if (e != cudaSuccess) {  // no bitmaps (speed only)
+      cudaGetLastError();
+      cudaFree(h.slot);
+      cudaFree(h.bits);
+      h.slot = nullptr;
+      h.bits = nullptr;
+      h.n_hubs = h.words = 0;
+    }
+  }
+  e = cudaMalloc(&h.vrec, sizeof(int4) * (size_t)std::max<int64_t>(n, 1));
+  if (e == cudaSuccess && n > 0) {
+    vrec_fill<<<grid, 256>>>(rp, n, ranked ? g->d_rout_start : g->d_out_start, h.slot, h.vrec);
     e = cudaGetLastError();
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
   }
   if (e != cudaSuccess) {
     cudaGetLastError();
-    free_hub(h);
-    h.min_deg = min_deg;
-    h.budget = budget;
+    cudaFree(h.vrec);
+    h.vrec = nullptr;
     return nullptr;
   }
-  h.words = words;
-  h.n_hubs = (int64_t)H;
   return &h;
 }
 
@@ -378,6 +412,8 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
   if (!row_ptr) return stm_fail(STM_EINVAL, "row_ptr is NULL");
   int64_t nnz = row_ptr[n];
   if (nnz > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
+  if (nnz > (int64_t)UINT32_MAX)  // packed vertex records hold 32-bit row starts (kernel.cu vrec)
+    return stm_fail(STM_EUNSUPPORTED, "%lld adjacency entries >= 2^32", (long long)nnz);
   stm_status s = validate_csr(n, row_ptr, col_idx);
   if (s != STM_OK) return s;
   std::vector<uint8_t> dense;
@@ -413,6 +449,7 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
                     cudaGetErrorString(e));
   }
+  g->has_stats = stm_graph_stats_host(n, row_ptr, labels, &g->stats) == STM_OK;
   build_ranked(g);
   g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
   if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
@@ -425,6 +462,13 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
                                             stm_graph** out) {
   if (!out || !d_row_ptr || (nnz > 0 && !d_col_idx)) return stm_fail(STM_EINVAL, "NULL argument");
   if (n < 0 || n > INT32_MAX - 1 || nnz < 0) return stm_fail(STM_EINVAL, "bad sizes");
+  if (nnz > (int64_t)UINT32_MAX)  // packed vertex records hold 32-bit row starts (kernel.cu vrec)
+    return stm_fail(STM_EUNSUPPORTED, "%lld adjacency entries >= 2^32", (long long)nnz);
+  {
+    int ndev = 0;
+    CU(cudaGetDeviceCount(&ndev));
+    if (device < 0 || device >= ndev) return stm_fail(STM_EINVAL, "device %d of %d", device, ndev);
+  }
   DeviceGuard dg(device);
   // cheap checks on the device: row_ptr[0] == 0, row_ptr[n] == nnz, monotone; max degree
   int64_t maxd = 0;
@@ -454,8 +498,9 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
   g->owns_csr = false;
   g->d_row_ptr = const_cast<int64_t*>(d_row_ptr);
   g->d_col_idx = const_cast<int32_t*>(d_col_idx);
+  std::vector<int32_t> lab;
   if (d_labels) {
-    std::vector<int32_t> lab(n);
+    lab.resize(n);
     cudaError_t e = cudaMemcpy(lab.data(), d_labels, sizeof(int32_t) * n, cudaMemcpyDeviceToHost);
     std::vector<uint8_t> dense;
     stm_status s = e == cudaSuccess ? dense_labels(n, lab.data(), dense, g->label_values)
@@ -473,6 +518,12 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
   cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
   cudaDeviceGetAttribute(&g->l2_bytes, cudaDevAttrL2CacheSize, device);
   query_persist(g);
+  {
+    std::vector<int64_t> rp(n + 1);
+    if (cudaMemcpy(rp.data(), d_row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost) == cudaSuccess)
+      g->has_stats = stm_graph_stats_host(n, rp.data(), d_labels ? lab.data() : nullptr, &g->stats) == STM_OK;
+    cudaGetLastError();
+  }
   build_ranked(g);
   g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
   if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
@@ -485,6 +536,13 @@ extern "C" stm_status stm_graph_info(const stm_graph* g, int64_t* n, int64_t* nn
   if (n) *n = g->n;
   if (nnz) *nnz = g->nnz;
   if (maxd) *maxd = g->max_degree;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_graph_get_stats(const stm_graph* g, stm_graph_stats* out) {
+  if (!g || !out) return stm_fail(STM_EINVAL, "NULL argument");
+  if (!g->has_stats) return stm_fail(STM_EUNSUPPORTED, "graph statistics unavailable");
+  *out = g->stats;
   return STM_OK;
 }
 
@@ -506,8 +564,7 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
   cudaFree(g->d_rlabels);
   cudaFree(g->d_out_start);
   cudaFree(g->d_rout_start);
-  free_hub(g->hub[0]);
-  free_hub(g->hub[1]);
+  for (auto& kv : g->hubs) free_hub(kv.second);
   delete g;
   return STM_OK;
 }
@@ -540,7 +597,7 @@ struct ListArgs {      // stm_match_list: root range and device output
 };
 
 static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tuning* tin,
-                         const stm_shard* shard, void* stream, uint64_t* d_count_out,
+                         const stm_shard* shard, void* stream, stm_async_result* d_result,
                          unsigned long long* d_per_root, uint64_t* h_count, ListArgs* la = nullptr) {
   if (!gc || !p) return stm_fail(STM_EINVAL, "NULL graph or plan");
   stm_graph* g = const_cast<stm_graph*>(gc);
@@ -553,6 +610,10 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.block_warps == 0) t.block_warps = 16;
   if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
   if (t.stop_level < 1) t.stop_level = 1;
+  if (t.watchdog_ms < 0) return stm_fail(STM_EINVAL, "watchdog_ms %d < 0", t.watchdog_ms);
+  if (t.backoff_max < 0 || t.backoff_max > 12) return stm_fail(STM_EINVAL, "backoff_max %d not in 0..12", t.backoff_max);
+  if (t.carveout_pct < -1 || t.carveout_pct > 100) return stm_fail(STM_EINVAL, "carveout_pct %d", t.carveout_pct);
+  if (d_result && ((uintptr_t)d_result & 7)) return stm_fail(STM_EINVAL, "d_result not 8-byte aligned");
   const StmPlan& P = p->dev;
   if (!p->labels.empty() && !g->d_labels) {
     bool any = false;
@@ -571,11 +632,10 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.plan = P;
   // order-free restrictions count on the degree-ranked copy (same count, less work)
   const bool use_rank = g->ranked && p->order_free && t.vertex_order == 0;
-  kp.row_ptr = use_rank ? g->d_rrow_ptr : g->d_row_ptr;
   kp.col_idx = use_rank ? g->d_rcol_idx : g->d_col_idx;
   kp.labels = use_rank ? g->d_rlabels : g->d_labels;
   kp.root_map = use_rank ? g->d_rank2orig : nullptr;
-  kp.out_start = t.narrow_split == 0 ? (use_rank ? g->d_rout_start : g->d_out_start) : nullptr;
+  kp.split = t.narrow_split == 0 ? 1 : 0;
   kp.n = g->n;
   if (la) {
     kp.root_lo = la->root_lo;
@@ -583,15 +643,16 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     kp.list_out = la->d_out;
     kp.list_cap = la->cap;
   }
+  std::unique_lock<std::mutex> glock(g->mu);  // per-numbering records / hub cache + L2 persistence state
   {
     const int min_deg = t.bitmap_min_degree == 0 ? STM_BITMAP_AUTO_MIN_DEGREE : t.bitmap_min_degree;
     const int64_t budget = (int64_t)(t.bitmap_budget_mb > 0 ? t.bitmap_budget_mb : STM_BITMAP_AUTO_BUDGET_MB) << 20;
-    std::lock_guard<std::mutex> lk(g->mu);
     const stm_graph::HubBitmaps* hb = ensure_hub(g, use_rank, min_deg, budget);
-    kp.hub_slot = hb ? hb->slot : nullptr;
-    kp.bitmaps = hb ? hb->bits : nullptr;
-    kp.bm_words = hb ? hb->words : 0;
-    g_info.hubs = hb ? hb->n_hubs : 0;
+    if (!hb) return stm_fail(STM_ENOMEM, "per-vertex records: %s", cudaGetErrorString(cudaGetLastError()));
+    kp.vrec = hb->vrec;
+    kp.bitmaps = hb->bits;
+    kp.bm_words = hb->words;
+    g_info.hubs = hb->n_hubs;
   }
   // label-slot table: dense graph label -> bitmask of pattern slots with that value
   for (int d = 0; d < (int)g->label_values.size(); ++d)
@@ -638,6 +699,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
       }
     }
   }
+  glock.unlock();
   kp.root_batch = std::max(1, std::min(STM_RMAX, root_chunk));
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
@@ -646,16 +708,15 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     return stm_fail(STM_EUNSUPPORTED, "hash_slots: this build has no hash-set path (-DSTM_WITH_HASH=1)");
   kp.ht_slots = t.hash_slots;
   kp.donate_mask = 0;  // look for idle blocks at every opportunity (measured: rate limiting starves idle blocks)
-  kp.backoff_max = 8;
+  kp.backoff_max = t.backoff_max ? t.backoff_max : 8;
   if (t.drive_ratio > 1 && !stm_drive_compiled())
     return stm_fail(STM_EUNSUPPORTED, "drive_ratio: this build has no drive-ratio path (-DSTM_DRIVE_RATIO=1)");
   kp.drive_ratio = t.drive_ratio;
-  if (const char* x = getenv("STM_DONATE_MASK")) kp.donate_mask = atoi(x);  // experiments
-  if (const char* x = getenv("STM_BACKOFF_MAX")) kp.backoff_max = atoi(x);
-  if (const char* wd = getenv("STM_WATCHDOG_S")) kp.watchdog_cycles = (long long)(atof(wd) * 2.0e9);
+  kp.watchdog_ns = (long long)t.watchdog_ms * 1000000LL;
+  kp.result = (unsigned long long*)d_result;
 
   int bps = 0;
-  int oe = (la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, &bps);
+  int oe = (la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy (variant %d, %s build, %d warps): %s", variant, la ? "list" : t.instrument ? "instr" : "count", t.block_warps, cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -717,18 +778,16 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   g_info.ranked = use_rank ? 1 : 0;
   g_info.variant = variant;
   g_info.unroll = kp.unroll;
-  if (d_count_out) {
-    CU(cudaMemcpyAsync(d_count_out, &work->count, sizeof(uint64_t), cudaMemcpyDeviceToDevice, st));
-  }
   if (h_count) {
     StmWork hw;
     CU(cudaMemcpyAsync(&hw, work, sizeof(StmWork), cudaMemcpyDeviceToHost, st));
     CU(cudaStreamSynchronize(st));
-    if (hw.overflow == 2) return stm_fail(STM_ECUDA, "watchdog expired (STM_WATCHDOG_S)");
+    if (hw.overflow == 2) return stm_fail(STM_ETIMEOUT, "launch aborted after watchdog_ms = %d", t.watchdog_ms);
     if (hw.overflow) return stm_fail(STM_EOVERFLOW, "device capacity exceeded");
     g_info.local_steals = (int64_t)hw.n_local_steals;
     g_info.global_steals = (int64_t)hw.n_global_steals;
     g_info.chunks = (int64_t)hw.n_chunks;
+    g_info.peer_chunks = (int64_t)hw.n_peer_chunks;
     g_info.alg_bytes = (int64_t)hw.alg_bytes;
     g_info.merge_bytes = (int64_t)hw.merge_bytes;
     g_info.jobs = (int64_t)hw.n_jobs;
@@ -753,9 +812,9 @@ extern "C" stm_status stm_match_count_ex(const stm_graph* g, const stm_plan* p, 
 }
 
 extern "C" stm_status stm_match_count_async(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
-                                            const stm_shard* shard, void* stream, uint64_t* d_count) {
-  if (!d_count) return stm_fail(STM_EINVAL, "d_count is NULL");
-  return launch(g, p, t, shard, stream, d_count, nullptr, nullptr);
+                                            const stm_shard* shard, void* stream, stm_async_result* d_result) {
+  if (!d_result) return stm_fail(STM_EINVAL, "d_result is NULL");
+  return launch(g, p, t, shard, stream, d_result, nullptr, nullptr);
 }
 
 extern "C" stm_status stm_match_count_per_root(const stm_graph* g, const stm_plan* p, const stm_tuning* t,
@@ -764,7 +823,11 @@ extern "C" stm_status stm_match_count_per_root(const stm_graph* g, const stm_pla
   DeviceGuard dg(g->device);
   unsigned long long* d = nullptr;
   CU(cudaMalloc(&d, sizeof(unsigned long long) * std::max<int64_t>(g->n, 1)));
-  cudaMemset(d, 0, sizeof(unsigned long long) * std::max<int64_t>(g->n, 1));
+  cudaError_t ze = cudaMemsetAsync(d, 0, sizeof(unsigned long long) * std::max<int64_t>(g->n, 1), (cudaStream_t)stream);
+  if (ze != cudaSuccess) {
+    cudaFree(d);
+    return stm_fail(STM_ECUDA, "per-root buffer: %s", cudaGetErrorString(ze));
+  }
   uint64_t c = 0;
   stm_status s = launch(g, p, t, nullptr, stream, nullptr, d, &c);
   if (s == STM_OK) {
@@ -820,5 +883,63 @@ extern "C" stm_status stm_last_profile(uint64_t* out, int n) {
 extern "C" stm_status stm_last_launch(stm_launch_info* info) {
   if (!info) return stm_fail(STM_EINVAL, "NULL info");
   *info = g_info;
+  return STM_OK;
+}
+
+// ---------------------------------------------------------------- IPC chunk cursors
+extern "C" stm_status stm_cursors_alloc(int device, int n_slots, uint64_t** d_base, void* ipc_handle) {
+  if (!d_base || !ipc_handle || n_slots < 1) return stm_fail(STM_EINVAL, "NULL argument or n_slots < 1");
+  int ndev = 0;
+  CU(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return stm_fail(STM_EINVAL, "device %d of %d", device, ndev);
+  static_assert(sizeof(cudaIpcMemHandle_t) <= STM_IPC_HANDLE_BYTES, "IPC handle size");
+  DeviceGuard dg(device);
+  void* d = nullptr;
+  const size_t bytes = (size_t)n_slots * 64;
+  CU(cudaMalloc(&d, bytes));
+  cudaError_t e = cudaMemset(d, 0, bytes);
+  cudaIpcMemHandle_t h;
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h, d);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) {
+    cudaFree(d);
+    return stm_fail(STM_ECUDA, "cursor allocation / IPC handle: %s", cudaGetErrorString(e));
+  }
+  memset(ipc_handle, 0, STM_IPC_HANDLE_BYTES);
+  memcpy(ipc_handle, &h, sizeof h);
+  *d_base = (uint64_t*)d;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_cursors_open(int device, const void* ipc_handle, uint64_t** d_peer_base) {
+  if (!ipc_handle || !d_peer_base) return stm_fail(STM_EINVAL, "NULL argument");
+  DeviceGuard dg(device);
+  cudaIpcMemHandle_t h;
+  memcpy(&h, ipc_handle, sizeof h);
+  void* d = nullptr;
+  CU(cudaIpcOpenMemHandle(&d, h, cudaIpcMemLazyEnablePeerAccess));
+  *d_peer_base = (uint64_t*)d;
+  return STM_OK;
+}
+
+extern "C" stm_status stm_cursors_close(int device, uint64_t* d_peer_base) {
+  if (!d_peer_base) return STM_OK;
+  DeviceGuard dg(device);
+  CU(cudaIpcCloseMemHandle(d_peer_base));
+  return STM_OK;
+}
+
+extern "C" stm_status stm_cursors_reset(int device, uint64_t* d_base, int first_slot, int n_slots,
+                                        void* stream) {
+  if (!d_base || first_slot < 0 || n_slots < 0) return stm_fail(STM_EINVAL, "bad cursor range");
+  DeviceGuard dg(device);
+  CU(cudaMemsetAsync((char*)d_base + (size_t)first_slot * 64, 0, (size_t)n_slots * 64, (cudaStream_t)stream));
+  return STM_OK;
+}
+
+extern "C" stm_status stm_cursors_free(int device, uint64_t* d_base) {
+  if (!d_base) return STM_OK;
+  DeviceGuard dg(device);
+  CU(cudaFree(d_base));
   return STM_OK;
 }

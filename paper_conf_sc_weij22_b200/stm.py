@@ -14,17 +14,20 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("STM_LIB_PATH") or os.path.join(_HERE, "libstm.so")  # override: A/B experiments only
 
-STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW = range(6)
+STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW, STM_ETIMEOUT = range(7)
 STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
 STM_LAZY_UNBOUNDED = 16
-_NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW"}
+_NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW",
+          6: "STM_ETIMEOUT"}
+STM_IPC_HANDLE_BYTES = 64
 
 EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_graph_info", "stm_graph_free",
            "stm_pattern_compile", "stm_plan_describe", "stm_plan_info", "stm_plan_free",
            "stm_plan_first_vertex", "stm_tuning_default", "stm_match_count", "stm_match_count_ex",
            "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error",
            "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize", "stm_motif_catalog",
-           "stm_motif_census"]
+           "stm_motif_census", "stm_cursors_alloc", "stm_cursors_open", "stm_cursors_close", "stm_cursors_free",
+           "stm_cursors_reset", "stm_graph_get_stats"]
 
 
 class StmError(RuntimeError):
@@ -38,7 +41,8 @@ class stm_tuning(ctypes.Structure):
                                                "unroll", "root_chunk", "block_warps", "blocks_per_sm",
                                                "instrument", "hash_slots", "vertex_order",
                                                "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
-                                               "l2_persist_mb", "drive_ratio", "narrow_split")]
+                                               "l2_persist_mb", "drive_ratio", "narrow_split", "watchdog_ms",
+                                               "backoff_max", "carveout_pct")]
 
 
 class stm_shard(ctypes.Structure):
@@ -52,7 +56,17 @@ class stm_launch_info(ctypes.Structure):
                 ("global_steals", ctypes.c_int64), ("chunks", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("merge_bytes", ctypes.c_int64), ("jobs", ctypes.c_int64), ("ranked", ctypes.c_int32),
                 ("reserved", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64),
-                ("hubs", ctypes.c_int64), ("variant", ctypes.c_int32), ("unroll", ctypes.c_int32)]
+                ("hubs", ctypes.c_int64), ("variant", ctypes.c_int32), ("unroll", ctypes.c_int32),
+                ("peer_chunks", ctypes.c_int64)]
+
+
+class stm_async_result(ctypes.Structure):
+    """Device-side result record of stm_match_count_async (4 x uint64)."""
+    _fields_ = [("count", ctypes.c_uint64), ("status", ctypes.c_uint64), ("chunks", ctypes.c_uint64),
+                ("peer_chunks", ctypes.c_uint64)]
+
+
+ASYNC_WORDS = 4  # uint64 words of stm_async_result
 
 
 STM_STATS_MOMENTS, STM_STATS_LABELS = 9, 256
@@ -92,6 +106,12 @@ def _load():
         "stm_motif_catalog": [i32, i32, vp, vp, ctypes.POINTER(i32)],
         "stm_motif_census": [vp, i32, u32, vp, vp, vp, i32, vp, ctypes.POINTER(i32)],
         "stm_graph_stats_host": [i64, vp, vp, ctypes.POINTER(stm_graph_stats)],
+        "stm_graph_get_stats": [vp, ctypes.POINTER(stm_graph_stats)],
+        "stm_cursors_alloc": [i32, i32, ctypes.POINTER(vp), vp],
+        "stm_cursors_open": [i32, vp, ctypes.POINTER(vp)],
+        "stm_cursors_close": [i32, vp],
+        "stm_cursors_free": [i32, vp],
+        "stm_cursors_reset": [i32, vp, i32, i32, vp],
         "stm_order_cost": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
                            ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
         "stm_order_optimize": [i32, i32, vp, vp, i32, vp, u32, ctypes.POINTER(stm_graph_stats), vp,
@@ -165,6 +185,12 @@ def stm_graph_stats_host(n: int, row_ptr, labels=None) -> stm_graph_stats:
     lb = _arr(labels, np.int32)
     st = stm_graph_stats()
     _check(lib.stm_graph_stats_host(n, _p(rp), _p(lb), ctypes.byref(st)))
+    return st
+
+
+def stm_graph_get_stats(g: int) -> stm_graph_stats:
+    st = stm_graph_stats()
+    _check(lib.stm_graph_get_stats(g, ctypes.byref(st)))
     return st
 
 
@@ -272,10 +298,42 @@ def stm_match_count_ex(g: int, p: int, tuning: Optional[stm_tuning] = None, shar
     return c.value
 
 
-def stm_match_count_async(g: int, p: int, d_count: int, tuning: Optional[stm_tuning] = None,
+def stm_match_count_async(g: int, p: int, d_result: int, tuning: Optional[stm_tuning] = None,
                           shard: Optional[stm_shard] = None, stream: Optional[int] = None) -> None:
+    """d_result: device address of an stm_async_result (4 x uint64, e.g. a torch int64[4] tensor)."""
     sp = None if shard is None else ctypes.cast(ctypes.pointer(shard), ctypes.c_void_p)
-    _check(lib.stm_match_count_async(g, p, _tp(tuning), sp, stream, d_count))
+    _check(lib.stm_match_count_async(g, p, _tp(tuning), sp, stream, d_result))
+
+
+def async_status_message(status: int) -> str:
+    return _NAMES.get(int(status), str(status))
+
+
+def stm_cursors_alloc(device: int, n_slots: int) -> Tuple[int, bytes]:
+    """n_slots zeroed device cursors (64 bytes apart) + their CUDA IPC handle bytes."""
+    d = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(STM_IPC_HANDLE_BYTES)
+    _check(lib.stm_cursors_alloc(device, n_slots, ctypes.byref(d), h))
+    return d.value, h.raw
+
+
+def stm_cursors_open(device: int, handle: bytes) -> int:
+    d = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(bytes(handle), STM_IPC_HANDLE_BYTES)
+    _check(lib.stm_cursors_open(device, h, ctypes.byref(d)))
+    return d.value
+
+
+def stm_cursors_close(device: int, d_peer: int) -> None:
+    _check(lib.stm_cursors_close(device, d_peer))
+
+
+def stm_cursors_reset(device: int, d_base: int, first_slot: int, n_slots: int, stream: Optional[int]) -> None:
+    _check(lib.stm_cursors_reset(device, d_base, first_slot, n_slots, stream))
+
+
+def stm_cursors_free(device: int, d_base: int) -> None:
+    _check(lib.stm_cursors_free(device, d_base))
 
 
 def stm_match_list(g: int, p: int, k: int, tuning: Optional[stm_tuning] = None, root_begin: int = 0,
@@ -353,9 +411,12 @@ class Plan:
 
     def __init__(self, k: int, edges, labels=None, order=None, restrictions=None, vertex_induced=False,
                  code_motion=True, auto_restrict=None, auto_order=False, lazy_unbounded=False,
-                 cost_stats: Optional[stm_graph_stats] = None):
+                 cost_stats: Optional[stm_graph_stats] = None, graph: Optional["Graph"] = None):
         """cost_stats: graph statistics (stm_graph_stats_host) -> the cost-optimal order (NEXT-2)
-        replaces `order`."""
+        replaces `order`.  graph: compile for this loaded graph -- its statistics (stm_graph_get_stats)
+        give the cost-based order unless `order` or `cost_stats` is given."""
+        if graph is not None and cost_stats is None and order is None and not auto_order:
+            cost_stats = stm_graph_get_stats(graph.handle)
         if auto_restrict is None:
             auto_restrict = restrictions is None
         flags = (STM_VERTEX_INDUCED if vertex_induced else 0) | (0 if code_motion else STM_NO_CODE_MOTION)

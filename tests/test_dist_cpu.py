@@ -102,3 +102,98 @@ def test_gloo_world2_partial_counts_all_reduce(steal):
         total, whole, exact_once = open(out).read().split()
     assert int(total) == int(whole) > 0
     assert exact_once == "1"
+
+
+# ---------------------------------------------------------------- cursor protocol
+def _simulate(world, nchunks, steps, seed, protocol):
+    """Discrete-event model of MultiGPUCounter's per-rank streams.  Each rank's stream is
+    [kernel(step) ; all-reduce(step) ; zero(own cursors of the step's set)] per step
+    ("new" protocol, dist.SlotSchedule), or [zero(own slot) ; kernel ; all-reduce] (the
+    round-1 protocol).  A kernel is a sequence of atomic fetch-adds, own cursor first then
+    the peers' (kernel try_chunk); an all-reduce completes on a rank only once every rank
+    has entered it.  The scheduler interleaves ranks at random.  Returns, per step, the
+    sorted list of chunks handed out."""
+    from paper_conf_sc_weij22_b200.dist import SlotSchedule
+    rng = np.random.default_rng(seed)
+    sched = [SlotSchedule(slots=1, sets=2) for _ in range(world)]
+    cursors = np.zeros((world, 2), np.int64)  # [owner, slot]
+    taken = [[] for _ in range(steps)]
+    # per-rank program counter: (step, phase, state)
+    ops = []
+    for r in range(world):
+        prog = []
+        for s in range(steps):
+            slot = sched[r].next_slot() if protocol == "new" else 0  # round 1: slot 0 every step
+            if protocol == "old":
+                prog.append(("zero", s, slot))
+            prog.append(("kernel", s, slot))
+            prog.append(("ar", s, slot))
+            if protocol == "new":
+                first, n = sched[r].end_step()
+                prog.append(("zero", s, first))
+        ops.append(prog)
+    pc = [0] * world
+    kstate = [None] * world  # exhausted set of the running kernel
+    entered_ar = [set() for _ in range(steps)]
+    speed = rng.random(world) ** 4 + 1e-3  # per-rank speed: some ranks far faster than others
+    while any(pc[r] < len(ops[r]) for r in range(world)):
+        def blocked(r):  # waiting inside an all-reduce that not every rank has entered
+            kind, s, _ = ops[r][pc[r]]
+            return kind == "ar" and r in entered_ar[s] and len(entered_ar[s]) < world
+        live = [r for r in range(world) if pc[r] < len(ops[r]) and not blocked(r)]
+        r = int(rng.choice(live, p=speed[live] / speed[live].sum()))  # skewed ranks
+        kind, s, slot = ops[r][pc[r]]
+        if kind == "zero":
+            cursors[r, slot] = 0
+            pc[r] += 1
+        elif kind == "ar":
+            entered_ar[s].add(r)
+            if len(entered_ar[s]) == world:  # completes for this rank only when all entered
+                pc[r] += 1
+        else:
+            if kstate[r] is None:
+                kstate[r] = set()
+            o = next((o for o in steal_order(r, world) if o not in kstate[r]), None)
+            if o is None:
+                kstate[r] = None
+                pc[r] += 1
+                continue
+            idx = int(cursors[o, slot])
+            cursors[o, slot] += 1
+            c = cursor_chunk(o, idx, world)
+            if c < nchunks:
+                taken[s].append(c)
+            else:
+                kstate[r].add(o)
+    return [sorted(t) for t in taken]
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_cursor_protocol_hands_out_every_chunk_once_per_step(world):
+    """dist.py's slot-set protocol: under any interleaving of the ranks' streams, every
+    step hands out every chunk exactly once (no chunk recounted after a reset, none lost)."""
+    for seed in range(60):
+        for t in _simulate(world, nchunks=23, steps=5, seed=seed, protocol="new"):
+            assert t == list(range(23))
+
+
+def test_cursor_protocol_round1_reset_race_is_caught():
+    """The round-1 order (each rank zeroes its own cursor right before its launch) recounts
+    chunks when a fast rank drains a slow rank's cursor first -- the model detects it."""
+    bad = 0
+    for seed in range(60):
+        bad += any(t != list(range(23)) for t in _simulate(2, nchunks=23, steps=5, seed=seed, protocol="old"))
+    assert bad > 0
+
+
+def test_slot_schedule_alternates_sets():
+    from paper_conf_sc_weij22_b200.dist import SlotSchedule
+    s = SlotSchedule(slots=4, sets=2)
+    assert [s.next_slot() for _ in range(3)] == [0, 1, 2]
+    assert s.end_step() == (0, 4)
+    assert s.next_slot() == 4
+    assert s.end_step() == (4, 4)
+    assert s.next_slot() == 0
+    with pytest.raises(RuntimeError):
+        for _ in range(5):
+            s.next_slot()

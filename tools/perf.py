@@ -1,12 +1,13 @@
 """Min-of-N timing of single queries through the C ABI: python tools/perf.py c2:k4,c2:c4,c5:k5 [key=val tuning...]"""
 import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-os.environ.setdefault("STM_WATCHDOG_S", "60")
+
 import stmgen
 from paper_conf_sc_weij22_b200 import stm
 specs = sys.argv[1].split(",")
 tk = dict(a.split("=") for a in sys.argv[2:] if "=" in a)
 reps = int(tk.pop("reps", 3))
+tk.setdefault("watchdog_ms", "60000")  # failure detection: a hung launch reports STM_ETIMEOUT
 graphs = {}
 for spec in specs:
     cfg, name = spec.split(":")[:2]
