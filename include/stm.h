@@ -63,6 +63,8 @@ enum {
   STM_NO_CODE_MOTION = 2,  /* recompute every level's candidate set from raw neighbour lists (ablation) */
   STM_AUTO_RESTRICT = 4,   /* ignore `restr`; use Grochow-Kellis symmetry-breaking restrictions */
   STM_AUTO_ORDER = 8,      /* ignore `order`; use the greedy connected order */
+  STM_CENSUS_PER_MOTIF = 32, /* stm_motif_census only: one counting launch per motif instead of the merged
+                                trie launch (A/B baseline of pattern merging) */
   STM_LAZY_UNBOUNDED = 16  /* code motion hoists only set chains that carry a restriction bound for their
                               consumer; a chain unbounded at its first operation is computed at the level
                               of its first consumer (no hoisting across levels whose prefixes rarely extend;
@@ -342,12 +344,15 @@ stm_status stm_last_launch(stm_launch_info* info);
 /*
  * stm_last_profile -- per-phase cycle buckets of this thread's last synchronous call,
  * filled only by libraries built with -DSTM_PROFILE=1 (A/B builds; zeros otherwise).
- * out receives min(n, 40) uint64: for phase i in 0..11 (root gather, root sibling
+ * out receives min(n, 114) uint64: for phase i in 0..11 (root gather, root sibling
  * set-up, candidate gather, set-node build, frame count, fused count, donate,
  * work acquisition, next-sibling set-up, descend set-up, combined-operation set-up,
  * combined-operation element loop) the triple (warp cycles, calls, items), then
  * the summed and the maximal warp lifetime, the summed and the maximal time (from
- * the warp's start) at which the root cursors were first seen exhausted.
+ * the warp's start) at which the root cursors were first seen exhausted; then for
+ * kind in (candidate pre-test, set build, count) and level 0..7 the triple (warp
+ * cycles, combined operations, driven elements); then the longest time one warp held a
+ * single task (root chunk or stolen work, cycles) and a reserved word.
  */
 stm_status stm_last_profile(uint64_t* out, int n);
 
@@ -434,14 +439,31 @@ stm_status stm_motif_catalog(int k, int capacity, int32_t* n_edges, int32_t* edg
  * induced k-vertex subsets), optionally | STM_NO_CODE_MOTION / STM_LAZY_UNBOUNDED.
  * stats: graph statistics (stm_graph_stats_host) to give each motif its cost-based
  * order (stm_order_optimize), or NULL for the graph's own statistics (stm_graph_get_stats);
- * flags | STM_AUTO_ORDER keeps the compiler's greedy order.  Counts are the same either way.  One counting launch per motif on `cuda_stream` (synchronous, as
- * stm_match_count_ex); t may be NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the
- * catalog size.  Errors: as stm_motif_catalog and stm_match_count_ex; STM_EINVAL for
- * other flag bits or a short capacity.
+ * flags | STM_AUTO_ORDER keeps the compiler's greedy order.  Counts are the same either way.
+ * Pattern merging: the motif plans are merged into one trie of matching
+ * levels -- motifs whose levels 0..d have the same candidate sources, filters and set-node
+ * definitions share one DFS frame and every set built on the way -- and the whole census
+ * is ONE persistent launch of the merged-plan kernel (a group whose merged plan exceeds
+ * the kernel's per-level limits is split into halves, one launch each;
+ * stm_motif_census_launches reports how many).  flags | STM_CENSUS_PER_MOTIF instead runs
+ * one counting launch per motif (the A/B baseline).  Synchronous on `cuda_stream`; t may be
+ * NULL (defaults).  counts: caller-owned uint64[capacity], capacity >= the catalog size.
+ * Errors: as stm_motif_catalog and stm_match_count_ex; STM_EINVAL for other flag bits or a
+ * short capacity.
  */
 stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags, const stm_graph_stats* stats,
                             const stm_tuning* t, void* cuda_stream, int capacity, uint64_t* counts,
                             int* n_motifs);
+
+/* stm_motif_census_launches -- counting launches of this thread's last stm_motif_census. */
+stm_status stm_motif_census_launches(int* launches);
+
+/*
+ * stm_motif_merge_stats -- shape of the merged trie of the size-k census (greedy orders,
+ * flags & STM_VERTEX_INDUCED): trie vertices per depth (int[k]), pool set nodes and
+ * per-warp set regions.  STM_EUNSUPPORTED when one merged launch cannot hold the census.
+ */
+stm_status stm_motif_merge_stats(int k, uint32_t flags, int* verts_per_depth, int* n_nodes, int* n_regions);
 
 /* stm_last_error -- thread-local message for the last non-OK status of this thread. */
 const char* stm_last_error(void);

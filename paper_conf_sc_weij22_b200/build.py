@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libstm.so")
-SOURCES = ["kernel.cu", "kernel_instr.cu", "kernel_list.cu", "runtime.cu", "compiler.cpp", "order.cpp", "motif.cpp"]
+SOURCES = ["kernel.cu", "kernel_instr.cu", "kernel_list.cu", "kernel_multi.cu", "runtime.cu", "compiler.cpp", "order.cpp", "motif.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

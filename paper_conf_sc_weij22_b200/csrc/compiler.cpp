@@ -361,7 +361,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
       prev = id;
     }
     cand_src[l].kind = (int8_t)prev_kind;
-    cand_src[l].idx = (int8_t)prev;
+    cand_src[l].idx = (int16_t)prev;
   }
 
   // ---- the final level is counted, never materialised (PAPER.md:75 Output at the
@@ -372,7 +372,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     const TNode& x = tn[last.idx];
     drop = last.idx;
     D.cnt_a.kind = (int8_t)x.a_kind;
-    D.cnt_a.idx = (int8_t)x.a;
+    D.cnt_a.idx = (int16_t)x.a;
     D.cnt_b = (int8_t)x.b;
     D.cnt_op = (int8_t)x.op;
     bool a_same_level = x.a_kind == STM_SRC_NODE && tn[x.a].level == k - 1;
@@ -407,7 +407,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     n.level = (int8_t)x.level;
     n.stage = (int8_t)stage[ids[i]];
     n.a_kind = (int8_t)x.a_kind;
-    n.a = (int8_t)(x.a_kind == STM_SRC_NODE ? remap[x.a] : x.a);
+    n.a = (int16_t)(x.a_kind == STM_SRC_NODE ? remap[x.a] : x.a);
     n.b = (int8_t)x.b;
     n.op = (int8_t)x.op;
     unsigned lm = 0, lo = 0xFF, hi = 0xFF;
@@ -436,9 +436,9 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   }
   for (int l = 1; l < k; ++l)
     if (cand_src[l].kind == STM_SRC_NODE && cand_src[l].idx != drop)
-      cand_src[l].idx = (int8_t)remap[cand_src[l].idx];
+      cand_src[l].idx = (int16_t)remap[cand_src[l].idx];
   for (int l = 1; l < k; ++l) D.cand[l] = cand_src[l];
-  if (D.cnt_a.kind == STM_SRC_NODE) D.cnt_a.idx = (int8_t)remap[D.cnt_a.idx];
+  if (D.cnt_a.kind == STM_SRC_NODE) D.cnt_a.idx = (int16_t)remap[D.cnt_a.idx];
   for (int l = 0; l < k; ++l) {
     D.filt[l].lab = (uint8_t)labmask(l);
     D.filt[l].lo = (uint8_t)reduce_lo(lo_pos[l]);

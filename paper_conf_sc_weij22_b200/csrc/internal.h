@@ -7,6 +7,7 @@
 #include <vector>
 
 #include "../../include/stm.h"
+#include "kernel.h"
 #include "plan.h"
 
 struct stm_plan {
@@ -23,3 +24,17 @@ struct stm_plan {
 
 // records a thread-local error message and returns the status
 stm_status stm_fail(stm_status s, const char* fmt, ...);
+
+// Merged multi-pattern plan (motif census, NEXT-3): host copy of the trie that
+// motif.cpp builds and runtime.cu uploads for the STM_MULTI kernel (kernel.h).
+struct stm_merged {
+  int k = 0;
+  int n_patterns = 0;
+  int n_regions = 0;                 // set-node storage regions per warp
+  std::vector<StmMVert> verts;       // the trie, children contiguous (BFS numbering)
+  std::vector<StmMNode> nodes;       // node pool
+  bool order_free = true;            // every pattern uses order-free (GK) restrictions
+};
+// one persistent launch of the merged plan; counts[i] += count of pattern i
+stm_status stm_launch_merged(const stm_graph* g, const stm_merged& m, const stm_tuning* t, void* stream,
+                             uint64_t* counts);

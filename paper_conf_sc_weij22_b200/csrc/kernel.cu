@@ -81,10 +81,15 @@
 #ifndef STM_LIST
 #define STM_LIST 0          // 1: the listing build (kernel_list.cu): last level emits embeddings (NEXT-1)
 #endif
+#ifndef STM_MULTI
+#define STM_MULTI 0         // 1: the merged-census build (kernel_multi.cu): a trie of patterns (NEXT-3)
+#endif
 #if STM_INSTR
 #define STM_SYM(x) x##_instr
 #elif STM_LIST
 #define STM_SYM(x) x##_list
+#elif STM_MULTI
+#define STM_SYM(x) x##_multi
 #else
 #define STM_SYM(x) x
 #endif
@@ -102,9 +107,20 @@
     w.prof_cnt[id] += 1;                                       \
     w.prof_items[id] += (unsigned long long)(items);           \
   }
+// per-level buckets: kind 0 pre-test, 1 set build, 2 count (level = the level computed)
+#define PROF_LVL_BEGIN() const long long prof_lt = clock64();
+#define PROF_LVL_END(kind, lvl)                                                                       \
+  if (w.lane == 0) {                                                                                \
+    unsigned long long* pl = &w.kp->work->prof[3 * STM_PROF_N + 4 + 3 * (8 * (kind) + (lvl))];        \
+    atomicAdd(pl, (unsigned long long)(clock64() - prof_lt));                                       \
+    atomicAdd(pl + 1, 1ull);                                                                        \
+    atomicAdd(pl + 2, (unsigned long long)w.last_total);                                            \
+  }
 #else
 #define PROF_BEGIN(id)
 #define PROF_END(id, items)
+#define PROF_LVL_BEGIN()
+#define PROF_LVL_END(kind, lvl)
 #endif
 
 namespace {
@@ -123,6 +139,11 @@ struct WarpHdr {
   int steal_fails;
   int pad0;
   long long first_dry;        // STM_PROFILE: clock64() when the root cursors were first seen exhausted
+  // STM_MULTI: frame F iterates the virtual siblings vs = child * nr[F] + u, u < nr[F]
+  // the real sibling (value of v_{F-1}) and child the child of trie vertex pv[F] whose
+  // candidates are enumerated (child-major: consecutive virtual siblings share a child,
+  // so the last level's counts pack up to 32 (sibling, candidate) pairs of one child)
+  int pv[STM_KMAX], nr[STM_KMAX];
 };
 
 struct BlockHdr {
@@ -159,6 +180,7 @@ struct W {
   unsigned long long idle_cyc;               // cycles in acquire_work (instrumented launches)
 #if STM_PROFILE
   unsigned long long prof_cyc[STM_PROF_N], prof_cnt[STM_PROF_N], prof_items[STM_PROF_N];
+  int last_total;  // elements driven by the last combined operation
 #endif
 };
 
@@ -251,19 +273,69 @@ __device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) 
 }
 __device__ __forceinline__ int degree(const W& w, int v) { return vrec(w, v).y; }
 
+// ----------------------------------------------------------------------------
+// plan access.  Single-pattern builds read the StmPlan; the STM_MULTI build reads the
+// merged trie (kernel.h StmMVert / StmMNode), where frame F's current sibling index
+// is virtual (real sibling * children + child).
+// ----------------------------------------------------------------------------
+#if STM_MULTI
+__device__ __forceinline__ const StmMVert& mvert(const W& w, int t) { return w.kp->mv[t]; }
+// trie vertex whose candidates frame F enumerates for virtual sibling vs
+__device__ __forceinline__ int vert_of(const W& w, int F, int vs) {
+  return F == 0 ? 0 : mvert(w, w.h->pv[F]).child_begin + vs / w.h->nr[F];
+}
+__device__ __forceinline__ StmSrc lvl_cand(const W& w, int F, int vs) { return mvert(w, vert_of(w, F, vs)).cand; }
+__device__ __forceinline__ StmFilter lvl_filt(const W& w, int F, int vs) { return mvert(w, vert_of(w, F, vs)).filt; }
+__device__ __forceinline__ int lvl_need(const W& w, int F, int vs) { return mvert(w, vert_of(w, F, vs)).need; }
+__device__ __forceinline__ const StmNode& pnode(const W& w, int s) { return w.kp->mn[s].nd; }
+__device__ __forceinline__ int pregion(const W& w, int s) { return w.kp->mn[s].region; }
+// pool nodes built after v_F is chosen from frame F's virtual sibling vs
+__device__ __forceinline__ void bset(const W& w, int F, int vs, int& b, int& e, int& nst) {
+  const StmMVert& t = mvert(w, vert_of(w, F, vs));
+  b = t.build_begin;
+  e = t.build_begin + t.n_build;
+  nst = t.n_stages;
+}
+#else
+__device__ __forceinline__ StmSrc lvl_cand(const W& w, int F, int) { return w.P->cand[F]; }
+__device__ __forceinline__ StmFilter lvl_filt(const W& w, int F, int) { return w.P->filt[F]; }
+__device__ __forceinline__ int lvl_need(const W& w, int F, int) { return w.P->need[F]; }
+__device__ __forceinline__ const StmNode& pnode(const W& w, int s) { return w.P->nodes[s]; }
+__device__ __forceinline__ int pregion(const W&, int s) { return s; }
+__device__ __forceinline__ void bset(const W& w, int F, int, int& b, int& e, int& nst) {
+  b = w.P->level_begin[F + 1];
+  e = w.P->level_begin[F + 2];
+  nst = w.P->n_stages[F + 1];
+}
+#endif
+// real sibling index of frame F's (virtual) sibling index vs
+#if STM_MULTI
+__device__ __forceinline__ int rsib(const W& w, int F, int vs) { return vs % w.h->nr[F]; }
+#else
+__device__ __forceinline__ int rsib(const W&, int, int vs) { return vs; }
+#endif
+
 // value of v_j in the context "frame F, sibling u, candidate c of level F"
 __device__ __forceinline__ int pval(const W& w, int j, int F, int u, int c) {
   if (j == F) return c;
-  if (j == F - 1) return SIB(w, F, u);
-  return SIB(w, j + 1, w.h->cur[j + 1]);
+  if (j == F - 1) return SIB(w, F, rsib(w, F, u));
+  return SIB(w, j + 1, rsib(w, j + 1, w.h->cur[j + 1]));
 }
 
 __device__ __forceinline__ void node_slice(const W& w, int s, int F, int u, int un, const int*& p,
                                            int& len) {
+#if STM_MULTI
+  const int lvl = pnode(w, s).level;
+  const int idx = lvl == F + 1 ? un : (lvl == F ? rsib(w, F, u) : rsib(w, lvl, w.h->cur[lvl]));
+  const int r = pregion(w, s);
+  p = w.arena + (size_t)r * w.kp->cap + NOFF(w, r, idx);
+  len = NSZ(w, r, idx);
+#else
   int lvl = w.P->nodes[s].level;
   int idx = lvl == F + 1 ? un : (lvl == F ? u : w.h->cur[lvl]);
   p = w.arena + (size_t)s * w.kp->cap + NOFF(w, s, idx);
   len = NSZ(w, s, idx);
+#endif
 }
 
 __device__ __forceinline__ void src_slice(const W& w, StmSrc src, int F, int u, int c, int un,
@@ -389,6 +461,9 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   }
   const int total = __shfl_sync(FULLMASK, incl, 31);
   const int start = incl - dlen;
+#if STM_PROFILE
+  w.last_total = total;
+#endif
   const int flags = (Pp != nullptr ? 1 : 0) | (J.op == STM_OP_DIFF ? 4 : 0) | (pslot >= 0 ? 8 : 0);
   const uint8_t* const glabels = w.kp->labels;
   const unsigned char* const l2s = w.bh->lab2slot;
@@ -512,8 +587,42 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   return s;
 }
 
+#if STM_MULTI
+// count job for the final level in context (F, u, c, un); lv = the leaf trie vertex
+// (STM_MULTI; ignored by single-pattern builds)
+__device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un, int lv = 0) {
+#if STM_MULTI
+  const StmMVert& L = mvert(w, lv);
+  const StmSrc ca = L.cand;
+  const int cb = L.cnt_b, cop = L.cnt_op;
+  const StmFilter f = L.filt;
+#else
+  (void)lv;
+  const StmPlan& P = *w.P;
+  const StmSrc ca = P.cnt_a;
+  const int cb = P.cnt_b, cop = P.cnt_op;
+  const StmFilter f = P.filt[P.k - 1];
+#endif
+  Job J;
+  if (ca.kind != STM_SRC_RAW) node_slice(w, ca.idx, F, u, un, J.A, J.alen);
+  J.B = nullptr;
+  J.blen = 0;
+  J.op = cop;
+  bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
+  J.abm = -1;
+  if (ca.kind == STM_SRC_RAW) row_narrow(w, pval(w, ca.idx, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+  J.bbm = -1;
+  if (cop != STM_OP_NONE) row_narrow(w, pval(w, cb, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+  J.lab = f.lab;
+  J.out = nullptr;
+  J.u = u;
+  J.c = c;
+  J.a_node = ca.kind == STM_SRC_NODE ? 1 : 0;
+  return J;
+}
+#else
 // count job for the final level in context (F, u, c, un)
-__device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un) {
+__device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un, int = 0) {
   const StmPlan& P = *w.P;
   Job J;
   if (P.cnt_a.kind != STM_SRC_RAW) node_slice(w, P.cnt_a.idx, F, u, un, J.A, J.alen);
@@ -531,9 +640,10 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   J.out = nullptr;
   J.u = u;
   J.c = c;
-  J.a_node = P.cnt_a.kind == STM_SRC_NODE ? P.nodes[P.cnt_a.idx].level + 1 : 0;
+  J.a_node = P.cnt_a.kind == STM_SRC_NODE ? 1 : 0;
   return J;
 }
+#endif
 
 // ----------------------------------------------------------------------------
 // locks and small helpers
@@ -564,7 +674,7 @@ __device__ __forceinline__ bool locked_frame(const W& w, int F) {
 __device__ __forceinline__ int src_len(const W& w, int F, int u) {
   const int* p;
   int len;
-  src_slice(w, w.P->cand[F], F, u, 0, 0, p, len);
+  src_slice(w, lvl_cand(w, F, u), F, u, 0, 0, p, len);
   return len;
 }
 
@@ -576,8 +686,8 @@ __device__ __forceinline__ int src_len(const W& w, int F, int u) {
 __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
   const int* p;
   int len;
-  src_slice(w, w.P->cand[F], F, u, 0, 0, p, len);
-  const StmFilter f = w.P->filt[F];
+  src_slice(w, lvl_cand(w, F, u), F, u, 0, 0, p, len);
+  const StmFilter f = lvl_filt(w, F, u);
   int b = 0, e = len;
   if ((f.lo | f.hi) && len > 0) {
     int lo, hi;
@@ -585,6 +695,7 @@ __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
     if (lo >= 0) b = lbound(p, len, lo + 1);
     if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
   }
+  if (e - b < lvl_need(w, F, u)) e = b;  // fewer candidates than any extension needs (plan.h need)
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->cur[F] = u;
@@ -596,7 +707,7 @@ __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
 
 // does candidate c (of level F, sibling u) pass the level's filter?
 __device__ __forceinline__ bool cand_ok(const W& w, int F, int u, int c, int lo, int hi) {
-  const StmFilter f = w.P->filt[F];
+  const StmFilter f = lvl_filt(w, F, u);
   if (!(c > lo && c < hi)) return false;
   if (!labok(w, c, f.lab)) return false;
   if (f.excl) {
@@ -608,13 +719,12 @@ __device__ __forceinline__ bool cand_ok(const W& w, int F, int u, int c, int lo,
 
 // upper bound on the size of node s (level F+1) for candidate c
 __device__ int node_ub(const W& w, int s, int F, int u, int c) {
-  const StmPlan& P = *w.P;
   int m = INT_MAX;
   for (;;) {
-    const StmNode nd = P.nodes[s];
+    const StmNode nd = pnode(w, s);
     if (nd.op == STM_OP_AND) m = min(m, degree(w, pval(w, nd.b, F, u, c)));
     if (nd.a_kind == STM_SRC_RAW) return min(m, degree(w, pval(w, nd.a, F, u, c)));
-    if (P.nodes[nd.a].level == F + 1) { s = nd.a; continue; }
+    if (pnode(w, nd.a).level == F + 1) { s = nd.a; continue; }
     const int* p;
     int len;
     node_slice(w, nd.a, F, u, 0, p, len);
@@ -625,13 +735,12 @@ __device__ int node_ub(const W& w, int s, int F, int u, int c) {
 // The part of node_ub that does not depend on the candidate (position F) of frame
 // F, sibling u: INT_MAX when every term does.
 __device__ int node_ub_const(const W& w, int s, int F, int u) {
-  const StmPlan& P = *w.P;
   int m = INT_MAX;
   for (;;) {
-    const StmNode nd = P.nodes[s];
+    const StmNode nd = pnode(w, s);
     if (nd.op == STM_OP_AND && nd.b != F) m = min(m, degree(w, pval(w, nd.b, F, u, 0)));
     if (nd.a_kind == STM_SRC_RAW) return nd.a != F ? min(m, degree(w, pval(w, nd.a, F, u, 0))) : m;
-    if (P.nodes[nd.a].level == F + 1) { s = nd.a; continue; }
+    if (pnode(w, nd.a).level == F + 1) { s = nd.a; continue; }
     const int* p;
     int len;
     node_slice(w, nd.a, F, u, 0, p, len);
@@ -651,11 +760,13 @@ __device__ __forceinline__ int compact_siblings(W& w, int F, int m, bool keep) {
   const int c = lane < m ? SIB(w, F + 1, lane) : 0;
   __syncwarp();
   if (mv) SIB(w, F + 1, dst) = c;
-  const StmPlan& P = *w.P;
-  for (int s = P.level_begin[F + 1]; s < P.level_begin[F + 2]; ++s) {
-    const int o = lane < m ? NOFF(w, s, lane) : 0, z = lane < m ? NSZ(w, s, lane) : 0;
+  int nb, ne, nst;
+  bset(w, F, w.h->cur[F], nb, ne, nst);
+  for (int s = nb; s < ne; ++s) {
+    const int r = pregion(w, s);
+    const int o = lane < m ? NOFF(w, r, lane) : 0, z = lane < m ? NSZ(w, r, lane) : 0;
     __syncwarp();
-    if (mv) { NOFF(w, s, dst) = o; NSZ(w, s, dst) = z; }
+    if (mv) { NOFF(w, r, dst) = o; NSZ(w, r, dst) = z; }
   }
   __syncwarp();
   return nm;
@@ -666,7 +777,103 @@ __device__ __forceinline__ int compact_siblings(W& w, int F, int m, bool keep) {
 // (plan.h need / pretest), siblings whose level-(F+1) candidate set cannot supply
 // need[F+1] candidates are dropped first (pre-test on bound-narrowed operands) or
 // after the build; returns the number of siblings kept.
+#if STM_MULTI
 __device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {
+  const int L1 = F + 1;
+  const int u = F >= 1 ? w.h->cur[F] : 0;
+  int nb, ne, nstages;
+  bset(w, F, u, nb, ne, nstages);
+  if (nb == ne) return m;
+#if STM_MULTI
+  prune = false;  // need / pretest are per pattern; the merged build serves every child
+  const StmFilter cf = {STM_LAB_ANY, 0, 0, 0};
+  const bool pre = false;
+  const int need1 = 1;
+  const StmSrc ccand = {STM_SRC_RAW, 0, 0};
+#else
+  const StmPlan& P = *w.P;
+  const bool pre = prune && P.pretest[L1];
+  const StmFilter cf = P.filt[L1];  // the candidate consumer's filter
+  const int need1 = P.need[L1];
+  const StmSrc ccand = P.cand[L1];
+#endif
+  // phase -1: candidate pre-test (probe counts); phases 0..: the level's stages.  The
+  // nodes of one stage are contiguous ([sb, se): ordered by stage).
+  int se = nb;
+  for (int st = pre ? -1 : 0; st < nstages; ++st) {
+    int sb = se;
+    if (st < 0) {
+      sb = ccand.idx;
+      se = sb + 1;
+    } else {
+      sb = st == 0 ? nb : se;
+      se = sb;
+      while (se < ne && pnode(w, se).stage == st) ++se;
+    }
+    const int njobs_total = (se - sb) * m;
+    for (int j0 = 0; j0 < njobs_total; j0 += 32) {
+      const int jj = j0 + w.lane;
+      const int nj = min(32, njobs_total - j0);
+      Job J;
+      J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_AND;
+      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
+      int r = 0, t = 0;
+      if (w.lane < nj) {
+        const int s = sb + jj / m;
+        t = jj % m;
+        r = pregion(w, s);
+        const StmNode nd = pnode(w, s);
+        const int c = SIB(w, L1, t);
+        J.c = c;
+        if (st < 0) bounds(w, cf.lo, cf.hi, F, u, c, J.lo, J.hi);  // the consumer's bounds
+        else bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
+        if (nd.a_kind == STM_SRC_RAW) row_narrow(w, pval(w, nd.a, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+        else node_slice(w, nd.a, F, u, t, J.A, J.alen);
+        J.a_node = nd.a_kind == STM_SRC_NODE ? 1 : 0;
+        row_narrow(w, pval(w, nd.b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+        J.op = nd.op;
+        J.lab = st < 0 ? cf.lab : nd.lab;
+        J.out = st < 0 ? nullptr : w.arena + (size_t)r * w.kp->cap + NOFF(w, r, t);
+      }
+      int outc = 0;
+      PROF_LVL_BEGIN()
+      run_jobs(w, J, nj, st < 0, F, 0, &outc, st < 0);
+      PROF_LVL_END(st < 0 ? 0 : 1, L1)
+      if (st < 0) {  // pre-test: one job per sibling (one node, m <= 32)
+        m = compact_siblings(w, F, m, outc >= need1);
+        if (m == 0) return 0;
+      } else {
+        if (w.lane < nj) NSZ(w, r, t) = outc;
+        __syncwarp();
+      }
+    }
+    if (st < 0) se = nb;  // the stages start at nb
+  }
+  // post-build check: a candidate node of this level smaller (within the consumer's
+  // bounds) than need[F+1] cannot be extended
+  if (prune && !pre && need1 > 1 && ccand.kind == STM_SRC_NODE && pnode(w, ccand.idx).level == L1) {
+    bool keep = true;
+    if (w.lane < m) {
+      const int c = SIB(w, L1, w.lane);
+      const int* p;
+      int len;
+      node_slice(w, ccand.idx, F, u, w.lane, p, len);
+      if (len >= need1 && (cf.lo | cf.hi)) {
+        int lo, hi;
+        bounds(w, cf.lo, cf.hi, F, u, c, lo, hi);
+        int b = 0, e = len;
+        if (lo >= 0) b = lbound(p, len, lo + 1);
+        if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
+        len = e - b;
+      }
+      keep = len >= need1;
+    }
+    m = compact_siblings(w, F, m, keep);
+  }
+  return m;
+}
+#else
+__device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {  // single-pattern plans
   const StmPlan& P = *w.P;
   const int L1 = F + 1;
   const int nb = P.level_begin[L1], ne = P.level_begin[L1 + 1];
@@ -709,7 +916,9 @@ __device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {
         J.out = st < 0 ? nullptr : w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
       }
       int outc = 0;
+      PROF_LVL_BEGIN()
       run_jobs(w, J, nj, st < 0, F, 0, &outc, st < 0);
+      PROF_LVL_END(st < 0 ? 0 : 1, L1)
       if (st < 0) {  // pre-test: one job per sibling (nn == 1, m <= 32)
         m = compact_siblings(w, F, m, outc >= P.need[L1]);
         if (m == 0) return 0;
@@ -743,6 +952,7 @@ __device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {
   }
   return m;
 }
+#endif
 
 // ----------------------------------------------------------------------------
 // gather: next batch of candidates of frame F (current sibling) as the
@@ -756,7 +966,7 @@ __device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* 
                                                  const int u) {
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0)
-    for (int s = nb; s < ne; ++s) w.h->used[s] = 0;
+    for (int s = nb; s < ne; ++s) w.h->used[s - nb] = 0;
   __syncwarp();
   int m = 0;
   bool cut = false;
@@ -775,7 +985,7 @@ __device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* 
         int t = __shfl_up_sync(FULLMASK, inc, o);
         if (w.lane >= o) inc += t;
       }
-      if (pass && w.h->used[s] + inc > cap) fits = false;
+      if (pass && w.h->used[s - nb] + inc > cap) fits = false;
     }
     unsigned pm = __ballot_sync(FULLMASK, pass);
     unsigned fm = __ballot_sync(FULLMASK, pass && fits);
@@ -803,11 +1013,11 @@ __device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* 
         int t = __shfl_up_sync(FULLMASK, inc, o);
         if (w.lane >= o) inc += t;
       }
-      int used = w.h->used[s];
-      if (me) NOFF(w, s, m + rank) = used + inc - ub;
+      int used = w.h->used[s - nb];
+      if (me) NOFF(w, pregion(w, s), m + rank) = used + inc - ub;
       int tot = __shfl_sync(FULLMASK, inc, 31);
       __syncwarp();
-      if (w.lane == 0) w.h->used[s] = used + tot;
+      if (w.lane == 0) w.h->used[s - nb] = used + tot;
       __syncwarp();
     }
     if (me) SIB(w, F + 1, m + rank) = c;
@@ -828,17 +1038,17 @@ __device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* 
 }
 
 __device__ STEP_INL int gather_batch(W& w, int F, int U) {
-  const StmPlan& P = *w.P;
   const int u = w.h->cur[F];
   const int* src;
   int len;
-  src_slice(w, P.cand[F], F, u, 0, 0, src, len);
+  src_slice(w, lvl_cand(w, F, u), F, u, 0, 0, src, len);
   int lo, hi;
-  const StmFilter f = P.filt[F];
+  const StmFilter f = lvl_filt(w, F, u);
   bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
   int pos = w.h->it[F];
   const int e = w.h->end[F];
-  const int nb = P.level_begin[F + 1], ne = P.level_begin[F + 2];
+  int nb, ne, nst;
+  bset(w, F, u, nb, ne, nst);
   const int cap = w.kp->cap;
   // Fast admission: when U copies of every node's candidate-independent size bound
   // fit in its region, any batch of <= U candidates fits -- fixed slice offsets
@@ -867,7 +1077,7 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
     }
     for (int s = nb; s < ne; ++s) {
       const int ub0 = node_ub_const(w, s, F, u);
-      if (w.lane < m) NOFF(w, s, w.lane) = w.lane * ub0;
+      if (w.lane < m) NOFF(w, pregion(w, s), w.lane) = w.lane * ub0;
     }
     HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) w.h->it[F] = pos;
@@ -879,14 +1089,14 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
 
 // root batch: up to root_batch roots from [root_it, root_end) with the root label
 __device__ int gather_roots(W& w) {
-  const StmPlan& P = *w.P;
+  const unsigned rlab = lvl_filt(w, 0, 0).lab;
   const int R = w.kp->root_batch;
   int pos = w.h->root_it;
   const int e = w.h->root_end;
   int m = 0;
   while (m < R && pos < e) {
     const int p = pos + w.lane;
-    const bool pass = p < e && labok(w, p, P.filt[0].lab);
+    const bool pass = p < e && labok(w, p, rlab);
     unsigned pm = __ballot_sync(FULLMASK, pass);
     int room = R - m;
     unsigned acc = pm;
@@ -918,12 +1128,26 @@ __device__ void frame_count(W& w, int m) {
   Job J;
   J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
   J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = u; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
+#if STM_MULTI
+  // every leaf (pattern) below the current trie vertex counts its final operation
+  const StmMVert& sv = mvert(w, vert_of(w, F, u));
+  for (int lv = sv.child_begin; lv < sv.child_begin + sv.n_children; ++lv) {
+    if (w.lane < m) J = count_job(w, F, u, SIB(w, k - 1, w.lane), w.lane, lv);
+    const unsigned long long c = run_jobs(w, J, m, true, F, mvert(w, lv).filt.excl, nullptr);
+    w.cnt += c;
+    if (w.lane == 0 && c) atomicAdd(&w.kp->mcount[mvert(w, lv).motif], c);
+  }
+#else
   if (w.lane < m) J = count_job(w, F, u, SIB(w, k - 1, w.lane), w.lane);
+  PROF_LVL_BEGIN()
   w.cnt += run_jobs(w, J, m, true, F, w.P->filt[k - 1].excl, nullptr);
+  PROF_LVL_END(2, k - 1)
+#endif
 }
 
 // fused mode at frame F = k-2: count over all remaining (sibling, candidate)
 // pairs, 32 jobs per pass.  Returns when the frame is exhausted.
+#if !STM_MULTI
 __device__ STEP_INL void fused_count(W& w, int F) {
   const StmPlan& P = *w.P;
   const bool lk = locked_frame(w, F);
@@ -982,10 +1206,88 @@ __device__ STEP_INL void fused_count(W& w, int F) {
     J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
     J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
     if (w.lane < nj) J = count_job(w, F, w.h->stage_u[w.lane], w.h->stage_c[w.lane], 0);
+    PROF_LVL_BEGIN()
     w.cnt += run_jobs(w, J, nj, true, F, P.filt[P.k - 1].excl, nullptr);
+    PROF_LVL_END(2, P.k - 1)
     __syncwarp();
   }
 }
+#endif  // !STM_MULTI
+
+#if STM_MULTI
+// Merged plans, last iterated frame F = k-2: while the current child builds no set node,
+// pack up to 32 (sibling, candidate) pairs of that child (consecutive virtual siblings,
+// child-major) and count every leaf below it over them.  Returns when the frame is
+// exhausted or reaches a child that needs level-(k-1) sets (the frame path builds those).
+__device__ STEP_INL void fused_count_multi(W& w, int F) {
+  const bool lk = locked_frame(w, F);
+  for (;;) {
+    if (lk) lock_ws(w, w.h);
+    int nj = 0, child = -1;
+    for (;;) {
+      const int u = w.h->cur[F];
+      if (u >= w.h->nsib[F]) break;
+      const int sv = vert_of(w, F, u);
+      if (mvert(w, sv).n_build != 0 || (child >= 0 && sv != child)) break;
+      child = sv;
+      const int pos = w.h->it[F], e = w.h->end[F];
+      if (pos >= e) {
+        if (u + 1 >= w.h->nsib[F]) {
+          HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+          if (w.lane == 0) w.h->cur[F] = u + 1;
+          __syncwarp();
+          break;
+        }
+        set_sibling(w, F, u + 1);
+        continue;
+      }
+      const int* src;
+      int len;
+      src_slice(w, lvl_cand(w, F, u), F, u, 0, 0, src, len);
+      const StmFilter f = lvl_filt(w, F, u);
+      int lo, hi;
+      bounds(w, f.lo, f.hi, F, u, 0, lo, hi);
+      const int p = pos + w.lane;
+      const bool valid = p < e;
+      const int c = valid ? src[p] : 0;
+      const bool pass = valid && cand_ok(w, F, u, c, lo, hi);
+      unsigned acc = __ballot_sync(FULLMASK, pass);
+      const int room = 32 - nj;
+      bool cut = false;
+      if (__popc(acc) > room) {
+        unsigned a2 = 0, t = acc;
+        for (int i = 0; i < room; ++i) { unsigned lsb = t & (0u - t); a2 |= lsb; t ^= lsb; }
+        acc = a2;
+        cut = true;
+      }
+      if ((acc >> w.lane) & 1u) {
+        const int r = nj + __popc(acc & ((1u << w.lane) - 1));
+        w.h->stage_c[r] = c;
+        w.h->stage_u[r] = u;
+      }
+      nj += __popc(acc);
+      const int npos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+      if (w.lane == 0) w.h->it[F] = npos;
+      __syncwarp();
+      if (nj == 32) break;
+    }
+    if (lk) unlock_ws(w, w.h);
+    if (nj == 0) return;
+    const StmMVert& sv = mvert(w, child);
+    for (int lv = sv.child_begin; lv < sv.child_begin + sv.n_children; ++lv) {
+      Job J;
+      J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
+      J.lo = -1; J.hi = INT_MAX; J.lab = STM_LAB_ANY; J.out = nullptr; J.u = 0; J.c = 0; J.a_node = 0; J.abm = -1; J.bbm = -1;
+      if (w.lane < nj) J = count_job(w, F, w.h->stage_u[w.lane], w.h->stage_c[w.lane], 0, lv);
+      const unsigned long long c = run_jobs(w, J, nj, true, F, mvert(w, lv).filt.excl, nullptr);
+      w.cnt += c;
+      if (w.lane == 0 && c) atomicAdd(&w.kp->mcount[mvert(w, lv).motif], c);
+    }
+    __syncwarp();
+  }
+}
+#endif
 
 // ----------------------------------------------------------------------------
 // work acquisition: root chunks, local steal, global steal (Sec. V)
@@ -1057,7 +1359,7 @@ __device__ __forceinline__ SplitPick pick_split(int stop, volatile WarpHdr* v) {
     const int cur = v->cur[F], nsib = v->nsib[F];
     if (cur >= nsib) continue;
     const int rem = v->end[F] - v->it[F];
-    if (F == 1) {
+    if (F == 1 && !STM_MULTI) {  // (merged plans: child-major frames have no whole-sibling split)
       const int rs = nsib - cur - 1;
       const int ts = (L > 1 || rem > 0) ? (rs + 1) / 2 : rs / 2;
       if (ts >= 1) return {1, 1, ts};
@@ -1090,7 +1392,13 @@ __device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr*
     T.level = F;
     T.e = v->end[F];
     T.b = v->end[F] - s.t;
+#if STM_MULTI
+    for (int j = 0; j < F; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1] % v->nr[j + 1]];
+    T.tv[0] = 0;
+    for (int d = 1; d <= F; ++d) T.tv[d] = (int16_t)(kp.mv[v->pv[d]].child_begin + v->cur[d] / v->nr[d]);
+#else
     for (int j = 0; j < F; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1]];
+#endif
     v->end[F] = T.b;
   }
   return true;
@@ -1155,19 +1463,30 @@ __device__ __noinline__ void adopt_task(const StmKParams& kp, const StmTask& T) 
     HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       SIB(w, i, 0) = T.prefix[i - 1];
+#if STM_MULTI
+      // the thief's frame i enumerates only the stolen path's child (virtual sibling ci)
+      const StmMVert& pv = kp.mv[T.tv[i - 1]];
+      const int ci = T.tv[i] - pv.child_begin;
+      w.h->pv[i] = T.tv[i - 1];
+      w.h->nr[i] = 1;
+      w.h->nsib[i] = ci + 1;
+      w.h->cur[i] = ci;
+#else
       w.h->nsib[i] = 1;
       w.h->cur[i] = 0;
+#endif
     }
     __syncwarp();
     if (i >= 2) {
-      const StmPlan& P = *w.P;
+      int nb, ne, nst;
+      bset(w, i - 1, w.h->cur[i - 1], nb, ne, nst);
       HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0)
-        for (int s = P.level_begin[i]; s < P.level_begin[i + 1]; ++s) NOFF(w, s, 0) = 0;
+        for (int s = nb; s < ne; ++s) NOFF(w, pregion(w, s), 0) = 0;
       __syncwarp();
       build_nodes(w, i - 1, 1, false);  // a stolen prefix is rebuilt as given
     }
-    int len = src_len(w, i, 0);
+    int len = src_len(w, i, w.h->cur[i]);
     HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->it[i] = (i == l) ? T.b : len;
@@ -1219,7 +1538,10 @@ __device__ __noinline__ bool try_local_steal(const StmKParams& kp) {
   T.level = bcast(T.level);
   T.b = bcast(T.b);
   T.e = bcast(T.e);
-  for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
+  for (int j = 0; j < STM_KMAX; ++j) {
+    T.prefix[j] = bcast(T.prefix[j]);
+    T.tv[j] = (int16_t)bcast(T.tv[j]);
+  }
   if (w.lane == 0) atomicAdd(&kp.work->n_local_steals, 1ull);
   adopt_task(kp, T);
   return true;
@@ -1270,7 +1592,10 @@ __device__ __noinline__ void maybe_donate(const StmKParams& kp) {
       M->level = T.level;
       M->b = T.b;
       M->e = T.e;
-      for (int j = 0; j < STM_KMAX; ++j) M->prefix[j] = T.prefix[j];
+      for (int j = 0; j < STM_KMAX; ++j) {
+        M->prefix[j] = T.prefix[j];
+        M->tv[j] = T.tv[j];
+      }
       __threadfence();
       atomicSub(&kp.work->idle_blocks, 1);
       __threadfence();
@@ -1340,7 +1665,10 @@ __device__ __noinline__ bool acquire_work(const StmKParams& kp, long long t0) {
           T.level = M->level;
           T.b = M->b;
           T.e = M->e;
-          for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = M->prefix[j];
+          for (int j = 0; j < STM_KMAX; ++j) {
+            T.prefix[j] = M->prefix[j];
+            T.tv[j] = M->tv[j];
+          }
           atomicExch(&S->mail_full, 0);
           atomicExch(&S->is_idle, 0);
           // leave the idle set before giving up leadership, so no other warp can
@@ -1352,7 +1680,10 @@ __device__ __noinline__ bool acquire_work(const StmKParams& kp, long long t0) {
         T.level = bcast(T.level);
         T.b = bcast(T.b);
         T.e = bcast(T.e);
-        for (int j = 0; j < STM_KMAX; ++j) T.prefix[j] = bcast(T.prefix[j]);
+        for (int j = 0; j < STM_KMAX; ++j) {
+          T.prefix[j] = bcast(T.prefix[j]);
+          T.tv[j] = (int16_t)bcast(T.tv[j]);
+        }
         adopt_task(kp, T);
         return true;
       }
@@ -1419,9 +1750,12 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
 
   const int k = P.k;
   const int U = max(1, min(kp.unroll, STM_UMAX));
-  const bool fused = P.count_mode == STM_COUNT_FUSED;
+  const bool fused = !STM_MULTI && P.count_mode == STM_COUNT_FUSED;
   const long long t0 = clock64();
   const long long wd0 = gtimer();
+#if STM_PROFILE
+  long long prof_task0 = clock64();
+#endif
   unsigned iter = 0;
   for (;;) {
     if ((++iter & 255) == 0 && watchdog(kp, wd0, "main")) break;
@@ -1435,7 +1769,13 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       if (m > 0) {
         // (reads above are ordered before this write by a full-warp collective)
         if (w.lane == 0) {
+#if STM_MULTI
+          w.h->pv[1] = 0;
+          w.h->nr[1] = m;
+          w.h->nsib[1] = m * kp.mv[0].n_children;
+#else
           w.h->nsib[1] = m;
+#endif
           w.h->cur[1] = 0;
         }
         __syncwarp();
@@ -1456,18 +1796,43 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
         // instrumented launches: time spent acquiring work (cursor, stealing, idle
         // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
         const long long ta = (STM_INSTR && kp.count_bytes) ? clock64() : 0;
+#if STM_PROFILE
+        // longest task (root chunk or stolen work) held by one warp: the critical path
+        if (lane == 0 && prof_task0) {
+          const unsigned long long d = (unsigned long long)(clock64() - prof_task0);
+          atomicMax(&kp.work->prof[3 * STM_PROF_N + 4 + STM_PROF_LVL - 2], d);
+        }
+#endif
         PROF_BEGIN(7)
         const bool got = acquire_work(kp, wd0);
         PROF_END(7, got)
+#if STM_PROFILE
+        prof_task0 = clock64();
+#endif
         if (STM_INSTR && kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
         if (!got) break;
       }
       continue;
     }
     const int F = L;
+#if STM_MULTI
+    if (F == k - 2 && mvert(w, vert_of(w, F, w.h->cur[F])).n_build == 0 && w.h->cur[F] < w.h->nsib[F]) {
+      fused_count_multi(w, F);
+      if (w.h->cur[F] < w.h->nsib[F]) continue;  // stopped at a child that builds sets
+      const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
+      if (lk) lock_ws(w, w.h);
+      // (reads above are ordered before this write by a full-warp collective)
+      if (w.lane == 0) w.h->L = F - 1;
+      if (lk) unlock_ws(w, w.h);
+      __syncwarp();
+      continue;
+    }
+#endif
     if (fused && F == k - 2) {
       PROF_BEGIN(5)
+#if !STM_MULTI
       fused_count(w, F);
+#endif
       PROF_END(5, 0)
       const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
       if (lk) lock_ws(w, w.h);
@@ -1478,7 +1843,9 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       continue;
     }
     const bool lk = locked_frame(w, F);
-    if (kp.global_steal && F < kp.detect_level && F < kp.stop_level) {
+    // donors look for idle blocks at frames < detect_level (they donate only work of
+    // frames < stop_level: pick_split)
+    if (kp.global_steal && F < kp.detect_level) {
       PROF_BEGIN(6)
       maybe_donate(kp);
       PROF_END(6, 0)
@@ -1489,8 +1856,16 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     for (;;) {
       if (w.h->cur[F] >= w.h->nsib[F]) { back = true; break; }
       if (w.h->it[F] < w.h->end[F]) {
+        int Ub = U;
+#if STM_MULTI
+        {  // a frame that builds no set node has no per-sibling slice table: batch up to 32
+          int nb, ne, nst;
+          bset(w, F, w.h->cur[F], nb, ne, nst);
+          if (nb == ne) Ub = STM_RMAX;
+        }
+#endif
         PROF_BEGIN(2)
-        m = gather_batch(w, F, U);
+        m = gather_batch(w, F, Ub);
         PROF_END(2, m)
         if (m > 0) break;
       }
@@ -1528,7 +1903,16 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     const bool lk2 = locked_frame(w, F + 1);
     if (lk2) lock_ws(w, w.h);
     // (reads above are ordered before this write by a full-warp collective)
-    if (w.lane == 0) w.h->nsib[F + 1] = m;
+    if (w.lane == 0) {
+#if STM_MULTI
+      const int sv = vert_of(w, F, w.h->cur[F]);
+      w.h->pv[F + 1] = sv;
+      w.h->nr[F + 1] = m;
+      w.h->nsib[F + 1] = m * kp.mv[sv].n_children;
+#else
+      w.h->nsib[F + 1] = m;
+#endif
+    }
     __syncwarp();
     PROF_BEGIN(9)
     set_sibling(w, F + 1, 0);
@@ -1596,19 +1980,28 @@ static const void* STM_SYM(kernel_fn)(int variant) {
   return variant == 2 ? (const void*)STM_SYM(stm_count_kernel_occ) : (const void*)STM_SYM(stm_count_kernel);
 }
 
-#if !STM_INSTR && !STM_LIST
+static int local_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
+  return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);
+}
+
+#if !STM_INSTR && !STM_LIST && !STM_MULTI
 int stm_drive_compiled() { return 0; }  // drive_ratio / hash sets: measured slower, removed
 int stm_hash_compiled() { return 0; }
 
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots) {
-  return (int)sizeof(BlockHdr) + block_warps * warp_bytes(k, n_nodes, ht_slots);
+  return local_smem_bytes(block_warps, k, n_nodes, ht_slots);
+}
+#endif
+#if STM_MULTI
+int stm_smem_bytes_multi(int block_warps, int k, int n_regions) {
+  return local_smem_bytes(block_warps, k, n_regions, 0);
 }
 #endif
 
 int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
                            int* blocks_per_sm) {
   const void* fn = STM_SYM(kernel_fn)(variant);
-  int smem = stm_smem_bytes(block_warps, k, n_nodes, ht_slots);
+  int smem = local_smem_bytes(block_warps, k, n_nodes, ht_slots);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   // The DFS stacks are the only shared-memory users: carve out just enough shared
@@ -1636,7 +2029,7 @@ int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int
 
 int STM_SYM(stm_launch)(int variant, const StmKParams& kp, int grid, void* stream) {
   const void* fn = STM_SYM(kernel_fn)(variant);
-  int smem = stm_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes, kp.ht_slots);
+  int smem = local_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes, kp.ht_slots);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
   void* args[] = {(void*)&kp};

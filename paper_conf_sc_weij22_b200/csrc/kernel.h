@@ -7,6 +7,32 @@
 
 #include "plan.h"
 
+// ---------------------------------------------------------------------------------
+// Merged multi-pattern plan (motif census; "pattern merging",
+// PAPER.md:25): the per-pattern plans are merged into a trie of matching levels.  A
+// trie vertex at depth d stands for every pattern whose levels 0..d are identical
+// (candidate source, filter, need, and the definitions of the set nodes they read);
+// its children are the distinct continuations.  The set nodes needed below a vertex
+// are built once per prefix when v_d is chosen (the union over its subtree, shared
+// by every pattern under it), and the leaves (depth k-1) carry each pattern's final
+// counting operation.  Built by motif.cpp, read by the STM_MULTI build of kernel.cu.
+struct StmMNode {     // a set node of the merged plan (StmNode fields + storage region)
+  StmNode nd;         // nd.a = pool index when nd.a_kind == STM_SRC_NODE
+  int16_t region;     // arena region / NOFF row of the node
+  int16_t pad;
+};
+struct StmMVert {
+  int16_t depth;
+  int16_t child_begin, n_children;   // children are vertices [child_begin, child_begin + n_children)
+  int16_t build_begin, n_build;      // pool nodes [build_begin, +n_build) of level depth+1, by stage
+  int8_t n_stages;
+  int8_t need;
+  StmSrc cand;                       // candidate source of level `depth` (leaves: the counted operand A)
+  StmFilter filt;                    // filter of level `depth`
+  int8_t cnt_b, cnt_op;              // leaves: count |A op N(v_cnt_b)|
+  int16_t motif;                     // leaves: pattern index (output slot)
+};
+
 // A unit of stealable work (Sec. V).  level 0: root-ID range
 // [b, e).  level l >= 1: the prefix v_0..v_{l-1} (prefix[0..l-1]) and the
 // positions [b, e) of the level-l candidate list of that prefix.  The candidate
@@ -17,6 +43,7 @@ struct StmTask {
   int32_t level;
   int32_t b, e;
   int32_t prefix[STM_KMAX];
+  int16_t tv[STM_KMAX];   // STM_MULTI: trie vertex of each level 0..level on the stolen path
 };
 
 // phases of the STM_PROFILE build: 0 gather_roots, 1 root set_sibling, 2 gather_batch,
@@ -24,6 +51,9 @@ struct StmTask {
 // 8 next-sibling set_sibling, 9 descend set_sibling, 10 run_jobs set-up (operand
 // narrowing), 11 run_jobs element loop (probes + compaction)
 #define STM_PROF_N 12
+// STM_PROFILE builds also keep, per level l (0..7) and kind (0 pre-test, 1 set build,
+// 2 count), the triple (warp cycles, combined operations, driven elements)
+#define STM_PROF_LVL (3 * 3 * 8 + 2)  // + (longest single task in cycles, its start time)
 
 // Device-resident scheduler state of one launch (zeroed before every launch).
 struct StmWork {
@@ -40,7 +70,7 @@ struct StmWork {
   unsigned long long idle_cycles;  // sum over warps of cycles spent acquiring work (instrumented)
   unsigned long long warp_cycles;  // sum over warps of their lifetime in cycles (instrumented)
   unsigned long long list_n;       // listing build: embeddings found (slots taken) so far
-  unsigned long long prof[3 * STM_PROF_N + 4];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
+  unsigned long long prof[3 * STM_PROF_N + 4 + STM_PROF_LVL];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
                                                 // lifetime, max lifetime, summed / max time cursors ran dry
 };
 
@@ -87,6 +117,10 @@ struct StmKParams {
   const void* l2_window_base;     // L2 persisting access-policy window (0 bytes = none)
   long long l2_window_bytes;
   uint8_t lab2slot[256];          // dense graph label -> pattern label-slot bitmask
+  // STM_MULTI (merged census) launches: the trie and node pool, per-pattern counts
+  const StmMVert* mv;
+  const StmMNode* mn;
+  unsigned long long* mcount;     // [n_patterns] counts (zeroed by the host)
 };
 
 // 1 if the shared-memory hash-set path is compiled in (-DSTM_WITH_HASH=1)
@@ -100,6 +134,7 @@ int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
 int stm_launch(int variant, const StmKParams& kp, int grid, void* stream);
 int stm_launch_instr(int variant, const StmKParams& kp, int grid, void* stream);  // instrumented build
 int stm_launch_list(int variant, const StmKParams& kp, int grid, void* stream);   // listing build
+int stm_launch_multi(int variant, const StmKParams& kp, int grid, void* stream);  // merged census build
 // max co-resident blocks per SM for the given block size
 // carveout: stm_tuning.carveout_pct (0 = auto, -1 = driver default, else percent)
 int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout, int* blocks_per_sm);
@@ -107,3 +142,6 @@ int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht
                         int* blocks_per_sm);
 int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
                        int* blocks_per_sm);
+int stm_occupancy_multi(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                        int* blocks_per_sm);
+int stm_smem_bytes_multi(int block_warps, int k, int n_regions);

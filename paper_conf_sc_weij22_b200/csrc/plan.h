@@ -36,13 +36,13 @@ struct StmNode {
   int8_t level;     // computed when entering this level
   int8_t stage;     // dependency stage within the level (0 = operands from earlier levels)
   int8_t a_kind;    // STM_SRC_NODE / STM_SRC_RAW
-  int8_t a;         // node index or level position of N(v_a)
   int8_t b;         // level position of N(v_b)
   int8_t op;        // STM_OP_AND / STM_OP_DIFF
   uint8_t lab;      // label-slot mask (STM_LAB_ANY = no label filter)
   uint8_t lo;       // bitmask of positions j: keep w > v_j
   uint8_t hi;       // bitmask of positions j: keep w < v_j
-  uint8_t pad[3];
+  int16_t a;        // node index (merged plans: pool index) or level position of N(v_a)
+  uint8_t pad[2];
 };
 
 // Candidate filter of one level: label, bounds, exclusions (injectivity for
@@ -53,8 +53,8 @@ struct StmFilter {
 
 struct StmSrc {
   int8_t kind;  // STM_SRC_NODE / STM_SRC_RAW
-  int8_t idx;   // node index or level position
-  int8_t pad[2];
+  int8_t pad;
+  int16_t idx;  // node index (merged plans: pool index) or level position
 };
 
 struct StmPlan {

@@ -27,7 +27,7 @@
 
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
-static thread_local uint64_t g_prof[3 * STM_PROF_N + 4] = {};
+static thread_local uint64_t g_prof[3 * STM_PROF_N + 4 + STM_PROF_LVL] = {};
 
 stm_status stm_fail(stm_status s, const char* fmt, ...) {
   va_list ap;
@@ -589,6 +589,12 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
 }
 
 // ---------------------------------------------------------------------------- match
+struct MultiArgs {     // merged census launch (STM_MULTI kernel build)
+  const StmMVert* d_verts = nullptr;
+  const StmMNode* d_nodes = nullptr;
+  unsigned long long* d_counts = nullptr;
+};
+
 struct ListArgs {      // stm_match_list: root range and device output
   int64_t root_lo = 0, root_hi = -1;
   int32_t* d_out = nullptr;
@@ -598,7 +604,8 @@ struct ListArgs {      // stm_match_list: root range and device output
 
 static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tuning* tin,
                          const stm_shard* shard, void* stream, stm_async_result* d_result,
-                         unsigned long long* d_per_root, uint64_t* h_count, ListArgs* la = nullptr) {
+                         unsigned long long* d_per_root, uint64_t* h_count, ListArgs* la = nullptr,
+                         const MultiArgs* ma = nullptr) {
   if (!gc || !p) return stm_fail(STM_EINVAL, "NULL graph or plan");
   stm_graph* g = const_cast<stm_graph*>(gc);
   stm_tuning t;
@@ -673,6 +680,12 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     variant = csr > (int64_t)g->l2_bytes / 2 ? 2 : 1;
   }
   kp.unroll = t.unroll ? t.unroll : (variant == 2 ? 32 : 16);
+  if (ma) {  // the merged build is compiled with 8 siblings per frame
+    kp.unroll = std::min(kp.unroll, 8);
+    kp.mv = ma->d_verts;
+    kp.mn = ma->d_nodes;
+    kp.mcount = ma->d_counts;
+  }
   const int root_chunk = t.root_chunk ? t.root_chunk : (variant == 2 ? 2 : 1);
   // root order: ascending by default -- descending (high-degree roots first on the
   // ranked copy) measured 1.2-1.7x slower on C2/C3 and neutral on C5
@@ -716,7 +729,9 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.result = (unsigned long long*)d_result;
 
   int bps = 0;
-  int oe = (la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps);
+  if (ma && (la || t.instrument)) return stm_fail(STM_EINVAL, "merged launches do not list or instrument");
+  int oe = (ma ? stm_occupancy_multi : la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(
+      variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy (variant %d, %s build, %d warps): %s", variant, la ? "list" : t.instrument ? "instr" : "count", t.block_warps, cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -768,11 +783,13 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   cudaStream_t st = (cudaStream_t)stream;
   CU(cudaMemsetAsync(S->state, 0, state_bytes, st));
-  int le = (la ? stm_launch_list : t.instrument ? stm_launch_instr : stm_launch)(variant, kp, grid, stream);
+  int le = (ma ? stm_launch_multi : la ? stm_launch_list : t.instrument ? stm_launch_instr : stm_launch)(
+      variant, kp, grid, stream);
   if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
   g_info.grid = grid;
   g_info.block_threads = t.block_warps * 32;
-  g_info.smem_bytes = stm_smem_bytes(t.block_warps, P.k, P.n_nodes, t.hash_slots);
+  g_info.smem_bytes = ma ? stm_smem_bytes_multi(t.block_warps, P.k, P.n_nodes)
+                         : stm_smem_bytes(t.block_warps, P.k, P.n_nodes, t.hash_slots);
   g_info.arena_bytes = (int64_t)arena_bytes;
   g_info.cap = kp.cap;
   g_info.ranked = use_rank ? 1 : 0;
@@ -874,9 +891,52 @@ extern "C" stm_status stm_match_list(const stm_graph* g, const stm_plan* p, cons
   return s;
 }
 
+stm_status stm_launch_merged(const stm_graph* g, const stm_merged& m, const stm_tuning* t, void* stream,
+                             uint64_t* counts) {
+  if (!g) return stm_fail(STM_EINVAL, "NULL graph");
+  DeviceGuard dg(g->device);
+  stm_plan tmp;  // the launch-shape view of the merged plan (k, set regions)
+  memset(&tmp.dev, 0, sizeof tmp.dev);
+  tmp.dev.k = m.k;
+  tmp.dev.n_nodes = m.n_regions;
+  tmp.dev.filt[0].lab = STM_LAB_ANY;
+  tmp.k = m.k;
+  tmp.order_free = m.order_free;
+  tmp.flags = STM_AUTO_RESTRICT;
+  MultiArgs ma;
+  void *dv = nullptr, *dn = nullptr, *dc = nullptr;
+  const size_t bv = sizeof(StmMVert) * std::max<size_t>(m.verts.size(), 1);
+  const size_t bn = sizeof(StmMNode) * std::max<size_t>(m.nodes.size(), 1);
+  const size_t bc = sizeof(unsigned long long) * std::max(m.n_patterns, 1);
+  cudaError_t e = cudaMalloc(&dv, bv);
+  if (e == cudaSuccess) e = cudaMalloc(&dn, bn);
+  if (e == cudaSuccess) e = cudaMalloc(&dc, bc);
+  if (e == cudaSuccess) e = cudaMemcpy(dv, m.verts.data(), sizeof(StmMVert) * m.verts.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess && !m.nodes.empty())
+    e = cudaMemcpy(dn, m.nodes.data(), sizeof(StmMNode) * m.nodes.size(), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemsetAsync(dc, 0, bc, (cudaStream_t)stream);
+  stm_status s = STM_OK;
+  if (e != cudaSuccess) s = stm_fail(STM_ECUDA, "merged plan upload: %s", cudaGetErrorString(e));
+  if (s == STM_OK) {
+    ma.d_verts = (const StmMVert*)dv;
+    ma.d_nodes = (const StmMNode*)dn;
+    ma.d_counts = (unsigned long long*)dc;
+    uint64_t total = 0;
+    s = launch(g, &tmp, t, nullptr, stream, nullptr, nullptr, &total, nullptr, &ma);
+    if (s == STM_OK) {
+      e = cudaMemcpy(counts, dc, sizeof(uint64_t) * m.n_patterns, cudaMemcpyDeviceToHost);
+      if (e != cudaSuccess) s = stm_fail(STM_ECUDA, "%s", cudaGetErrorString(e));
+    }
+  }
+  cudaFree(dv);
+  cudaFree(dn);
+  cudaFree(dc);
+  return s;
+}
+
 extern "C" stm_status stm_last_profile(uint64_t* out, int n) {
   if (!out || n < 0) return stm_fail(STM_EINVAL, "NULL out");
-  for (int i = 0; i < n && i < 3 * STM_PROF_N + 4; ++i) out[i] = g_prof[i];
+  for (int i = 0; i < n && i < 3 * STM_PROF_N + 4 + STM_PROF_LVL; ++i) out[i] = g_prof[i];
   return STM_OK;
 }
 

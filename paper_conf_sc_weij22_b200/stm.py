@@ -17,6 +17,7 @@ LIB_PATH = os.environ.get("STM_LIB_PATH") or os.path.join(_HERE, "libstm.so")  #
 STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW, STM_ETIMEOUT = range(7)
 STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
 STM_LAZY_UNBOUNDED = 16
+STM_CENSUS_PER_MOTIF = 32
 _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW",
           6: "STM_ETIMEOUT"}
 STM_IPC_HANDLE_BYTES = 64
@@ -27,7 +28,7 @@ EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_gra
            "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error",
            "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize", "stm_motif_catalog",
            "stm_motif_census", "stm_cursors_alloc", "stm_cursors_open", "stm_cursors_close", "stm_cursors_free",
-           "stm_cursors_reset", "stm_graph_get_stats"]
+           "stm_cursors_reset", "stm_graph_get_stats", "stm_motif_census_launches", "stm_motif_merge_stats"]
 
 
 class StmError(RuntimeError):
@@ -105,6 +106,8 @@ def _load():
         "stm_last_launch": [ctypes.POINTER(stm_launch_info)],
         "stm_motif_catalog": [i32, i32, vp, vp, ctypes.POINTER(i32)],
         "stm_motif_census": [vp, i32, u32, vp, vp, vp, i32, vp, ctypes.POINTER(i32)],
+        "stm_motif_census_launches": [ctypes.POINTER(i32)],
+        "stm_motif_merge_stats": [i32, u32, vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
         "stm_graph_stats_host": [i64, vp, vp, ctypes.POINTER(stm_graph_stats)],
         "stm_graph_get_stats": [vp, ctypes.POINTER(stm_graph_stats)],
         "stm_cursors_alloc": [i32, i32, ctypes.POINTER(vp), vp],
@@ -242,6 +245,19 @@ def stm_motif_census(g: int, k: int, flags: int = 0, stats: Optional[stm_graph_s
     return [int(x) for x in out[: n.value]]
 
 
+def stm_motif_census_launches() -> int:
+    n = ctypes.c_int()
+    _check(lib.stm_motif_census_launches(ctypes.byref(n)))
+    return n.value
+
+
+def stm_motif_merge_stats(k: int, flags: int = 0) -> dict:
+    per = np.zeros(k, np.int32)
+    nn, nr = ctypes.c_int(), ctypes.c_int()
+    _check(lib.stm_motif_merge_stats(k, flags, _p(per), ctypes.byref(nn), ctypes.byref(nr)))
+    return {"verts_per_depth": per.tolist(), "pool_nodes": nn.value, "regions": nr.value}
+
+
 def stm_plan_describe(p: int) -> str:
     buf = ctypes.create_string_buffer(1 << 16)
     _check(lib.stm_plan_describe(p, buf, len(buf)))
@@ -366,12 +382,21 @@ PROF_PHASES = ["gather_roots", "root_sibling", "gather_batch", "build_nodes", "f
 
 def stm_last_profile() -> dict:
     N = 3 * len(PROF_PHASES) + 4
-    out = (ctypes.c_uint64 * N)()
-    _check(lib.stm_last_profile(out, N))
+    NL = 3 * 3 * 8 + 2
+    out = (ctypes.c_uint64 * (N + NL))()
+    _check(lib.stm_last_profile(out, N + NL))
     d = {ph: {"cycles": out[3 * i], "calls": out[3 * i + 1], "items": out[3 * i + 2]}
          for i, ph in enumerate(PROF_PHASES)}
     d["lifetime_cycles"] = out[N - 4]
     d["tail"] = {"max_lifetime": out[N - 3], "sum_dry": out[N - 2], "max_dry": out[N - 1]}
+    lv = {}
+    for kind, kn in enumerate(["pretest", "build", "count"]):
+        for lvl in range(8):
+            c, j, e = out[N + 3 * (8 * kind + lvl):N + 3 * (8 * kind + lvl) + 3]
+            if j:
+                lv[f"{kn}@L{lvl}"] = {"cycles": c, "ops": j, "elements": e}
+    d["levels"] = lv
+    d["max_task_cycles"] = out[N + NL - 2]
     return d
 
 

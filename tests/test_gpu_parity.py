@@ -194,35 +194,40 @@ def test_golden_config_counts():
         assert stm.count(G, plan2) == d["count"], cid + " (compiler's own restrictions)"
 
 
-@pytest.mark.parametrize("cfg,name,ntop", [("c2", "k4", 1), ("c2", "c4", 0), ("c4", "house", 0), ("c5", "k5", 1),
-                                           ("c3", "k5", 0)])
-def test_config_scale_sampled_roots(cfg, name, ntop):
-    """At full size, in the bench's launch configuration: GPU per-root counts on a
-    sample of roots (random + the highest-degree ones) equal the oracle's."""
+def stratified_roots(n, sizes, seed=5):
+    """Degree-stratified root sample of a degree-ranked graph (vertex i = i-th lowest degree):
+    `sizes` roots from ranks [0, n-4096), [n-4096, n-256), [n-256, n-16), [n-16, n)."""
+    rng = np.random.default_rng(seed)
+    cuts = [0, max(0, n - 4096), max(0, n - 256), max(0, n - 16), n]
+    out = [rng.choice(np.arange(a, b), size=min(k, b - a), replace=False)
+           for (a, b), k in zip(zip(cuts[:-1], cuts[1:]), sizes) if b > a and k]
+    return np.unique(np.concatenate(out))
+
+
+@pytest.mark.parametrize("cfg,name,sizes", [
+    ("c5", "k5", (24, 8, 4, 2)), ("c5", "k6_minus_e", (24, 8, 1, 0)),
+    ("c3", "house", (24, 2, 0, 0)), ("c3", "c5", (24, 2, 0, 0)), ("c3", "k5", (24, 8, 4, 2)),
+    ("c2", "c4", (24, 8, 2, 0)), ("c2", "k4", (24, 8, 4, 2))])
+def test_config_scale_sampled_roots(cfg, name, sizes):
+    """At full size, in the bench's launch configuration (degree-ranked copy, default
+    tuning): GPU per-root counts on a degree-stratified sample of roots -- the bulk, the
+    high-degree strata where the work concentrates, and (where the oracle can afford them)
+    the top hubs -- equal the oracle's, run on the same graph renumbered in (degree, id)
+    order with matches attributed to f(order[0]) as on the GPU.  The sample must hold
+    matches (no zero-versus-zero pass)."""
     g = stmgen.config_graph(cfg)
     G = stm.Graph.from_stmgen(g)
     p = CATALOG[name]
     plan = stm.Plan(p.k, p.edges)
     R = oracle.gk_restrictions(p.k, p.edges)
-    rng = np.random.default_rng(5)
-    deg = g.degrees()
-    # caller's numbering (vertex_order=1)
-    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(vertex_order=1))
-    assert int(pr.sum(dtype=np.uint64)) == tot
-    top = np.argsort(deg)[len(deg) - ntop:] if ntop else np.zeros(0, np.int64)
-    roots = np.unique(np.concatenate([rng.choice(g.n, 48, replace=False), top]))
-    oc, opr = oracle.count(g, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=roots, per_root=True)
-    assert np.array_equal(pr[roots], opr)
-    # default: degree-ranked symmetry breaking, as bench.py times it; the oracle runs on
-    # the graph renumbered in (degree, id) order
-    tot2, pr2 = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
+    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
     assert stm.stm_last_launch()["ranked"] == 1
-    assert tot2 == tot and int(pr2.sum(dtype=np.uint64)) == tot
+    assert int(pr.sum(dtype=np.uint64)) == tot
     rank2orig, gr = degree_ranked(g)
-    rroots = np.unique(np.concatenate([rng.choice(g.n, 48, replace=False), np.arange(g.n - ntop, g.n)]))
-    oc2, opr2 = oracle.count(gr, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=rroots,
-                             per_root=True)
-    assert np.array_equal(pr2[rank2orig[rroots]], opr2)
+    roots = stratified_roots(g.n, sizes)
+    oc, opr = oracle.count(gr, p.k, p.edges, restrictions=R, root_u=plan.first_vertex, roots=roots, per_root=True)
+    assert np.array_equal(pr[rank2orig[roots]], opr)
+    assert int(opr.sum()) > 0 and np.count_nonzero(opr) >= 2, "sample holds no matches"
 
 
 def degree_ranked(g):
@@ -400,16 +405,40 @@ def test_cost_order_counts(rmat_small, name, vi):
 @pytest.mark.parametrize("k", [3, 4, 5])
 @pytest.mark.parametrize("vi", [False, True])
 def test_motif_census(rmat_small, k, vi):
-    """NEXT-3: every motif of the size-k catalog, bit-exact against the oracle."""
+    """NEXT-3: every motif of the size-k catalog, bit-exact against the oracle -- merged
+    (pattern merging: one launch of the trie plan) and per motif, greedy and
+    cost-based orders, with stealing off and forced (root chunk 1, deep stop level)."""
     g, G = rmat_small
     flags = stm.STM_VERTEX_INDUCED if vi else 0
     got = stm.stm_motif_census(G.handle, k, flags)
+    if k >= 3:
+        assert stm.stm_motif_census_launches() == 1
     cat = stm.stm_motif_catalog(k)
     assert len(got) == len(cat)
-    stats = stm.stm_graph_stats_host(g.n, g.row_ptr)
-    assert stm.stm_motif_census(G.handle, k, flags, stats) == got
     for edges, c in zip(cat, got):
         assert c == oracle.count(g, k, edges, vertex_induced=vi, restrictions=oracle.gk_restrictions(k, edges))
+    assert stm.stm_motif_census(G.handle, k, flags | stm.STM_CENSUS_PER_MOTIF) == got
+    assert stm.stm_motif_census_launches() == len(cat)
+    assert stm.stm_motif_census(G.handle, k, flags | stm.STM_AUTO_ORDER) == got
+    stats = stm.stm_graph_stats_host(g.n, g.row_ptr)
+    assert stm.stm_motif_census(G.handle, k, flags, stats) == got
+    for tk in (dict(local_steal=0, global_steal=0), dict(root_chunk=1, stop_level=4, detect_level=4, unroll=3),
+               dict(vertex_order=1, block_warps=4)):
+        assert stm.stm_motif_census(G.handle, k, flags, tuning=stm.stm_tuning_default(**tk)) == got, tk
+
+
+@pytest.mark.parametrize("vi", [False, True])
+def test_motif_census_k6_merged(vi):
+    """The 112-motif size-6 census in one merged launch, bit-exact against the oracle."""
+    g = stmgen.er(90, 330, 31)
+    G = stm.Graph.from_stmgen(g)
+    flags = stm.STM_VERTEX_INDUCED if vi else 0
+    got = stm.stm_motif_census(G.handle, 6, flags)
+    assert stm.stm_motif_census_launches() == 1
+    cat = stm.stm_motif_catalog(6)
+    want = [oracle.count(g, 6, e, vertex_induced=vi, restrictions=oracle.gk_restrictions(6, e)) for e in cat]
+    assert got == want
+    assert sum(got) > 0
 
 
 def test_motif_census_sums_to_connected_subsets():

@@ -37,12 +37,17 @@ for spec in specs:
         if prof["lifetime_cycles"]:
             L = prof.pop("lifetime_cycles")
             tail = prof.pop("tail")
+            lv = prof.pop("levels")
+            mt = prof.pop("max_task_cycles")
+            print(f"   longest single task (critical path): {mt / 1.9e6:.2f} ms", flush=True)
             nw = info["grid"] * info["block_threads"] // 32
             print(f"   tail: mean lifetime {L / nw / 1.9e6:.2f} ms, max {tail['max_lifetime'] / 1.9e6:.2f} ms, "
                   f"cursors dry at mean {tail['sum_dry'] / nw / 1.9e6:.2f} ms / max {tail['max_dry'] / 1.9e6:.2f} ms "
                   f"(1.9 GHz)", flush=True)
             print("   profile: " + "  ".join(f"{k}={100.0 * v['cycles'] / L:.1f}%/{v['calls']}/{v['items']}"
                                            for k, v in prof.items() if v["calls"]), flush=True)
+            print("   levels: " + "  ".join(f"{k}={100.0 * v['cycles'] / L:.1f}%/{v['ops']}/{v['elements']}"
+                                          for k, v in lv.items()), flush=True)
         print(f"{spec:16} {tk} count {c:>16} best {best*1e3:9.2f} ms  {c/best:.3e} m/s  ls={info['local_steals']} gs={info['global_steals']} grid={info['grid']} smem={info['smem_bytes']}", flush=True)
     except Exception as e:
         print(f"{spec:16} {tk} ERR {e}", flush=True)
