@@ -57,8 +57,7 @@ PER_CONFIG = [
     ("c1", "triangle", False, None),
     ("c2", "k4", False, None), ("c2", "c4", False, None), ("c2", "c4", True, None),
     ("c3", "k5", False, None), ("c3", "k5", True, None), ("c3", "c5", False, None),
-    ("c4", "c6", False, (0, 1, 2, 0, 1, 2)), ("c4", "prism", False, (0, 0, 1, 0, 0, 1)),
-    ("c4", "c7", False, (0, 1, 2, 3, 0, 1, 2)), ("c4", "w6", False, (0, 1, 1, 1, 1, 1, 1)),
+    ("c4", "c6", False, (0, 1, 2, 0, 1, 2)), ("c4", "c6", False, (0, 1, 2, 3, 4, 5)),
     ("c4", "c6", True, (0, 1, 2, 0, 1, 2)), ("c4", "c7", True, (0, 1, 2, 3, 0, 1, 2)),
 ]
 # The oracle counts K6-e through an isomorphic labelling whose non-adjacent pair is (4, 5):

@@ -195,6 +195,11 @@ typedef struct stm_tuning {
   int32_t carveout_pct;   /* shared-memory carveout of the unified L1/shared array in percent: 0 = auto
                              (just enough for the resident DFS stacks, rest to L1), -1 = driver default,
                              else 1..100.  Speed only. */
+  int32_t root_split;     /* root splitting: a root of degree d is handed out as ceil(d / root_split)
+                             independent pieces, piece c enumerating positions [c*root_split,
+                             (c+1)*root_split) of its level-1 candidate list, so the heaviest roots are
+                             spread over many warps from the start instead of being split by stealing.
+                             0 = auto (512), -1 = off (one piece per root).  Speed only. */
 } stm_tuning;
 
 /* Fill t with the defaults. */

@@ -144,6 +144,7 @@ struct WarpHdr {
   // candidates are enumerated (child-major: consecutive virtual siblings share a child,
   // so the last level's counts pack up to 32 (sibling, candidate) pairs of one child)
   int pv[STM_KMAX], nr[STM_KMAX];
+  int rent[STM_RMAX];         // root entries (kp.entries): entry index of frame-1 sibling u
 };
 
 struct BlockHdr {
@@ -442,12 +443,23 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
     // ceil(log2 |P|) dependent loads (the driving element already lies in (lo, hi))
     if (pslot >= 0) Pp = (const int*)(w.kp->bitmaps + (size_t)pslot * (size_t)w.kp->bm_words);
   }
+  // A counted set with no probe operand and no label filter is a bounded view: its
+  // count is the narrowed length (narrowing is exact once that exceeds 16), no element
+  // is visited -- the last level of K6-e / stars / paths is O(log) per job instead of
+  // O(|A|) (the exclusion correction below still applies).
+  unsigned long long jc0 = 0;
+  if (!STM_LIST && count_mode && !probe && mine && !J.B && J.lab == STM_LAB_ANY && an > 16) {
+    jc0 = (unsigned long long)an;
+    dlen = 0;
+  }
   if (STM_INSTR && w.kp->count_bytes && mine) {
     // W_op = 4|A| + 4 min(|B|, |A| ceil(log2(|B|+1))) (+ 4|out| below),
-    // with A the driving operand and B the probed one (before hashing).
+    // with A the driving operand and B the probed one (before hashing); a counted
+    // bounded view moves only its two bound searches
     int d, pl;
     if (J.op == STM_OP_AND) { d = min(an, bn); pl = max(an, bn); } else { d = an; pl = bn; }
-    w.wbytes += 4ull * (unsigned long long)d + 4ull * (unsigned long long)min((long long)pl, (long long)d * log2c(pl));
+    if (jc0) w.wbytes += 8ull * (unsigned long long)log2c(J.alen);
+    else w.wbytes += 4ull * (unsigned long long)d + 4ull * (unsigned long long)min((long long)pl, (long long)d * log2c(pl));
     w.wmerge += 4ull * (unsigned long long)(an + bn);
     w.wjobs += 1;
   }
@@ -468,7 +480,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   const uint8_t* const glabels = w.kp->labels;
   const unsigned char* const l2s = w.bh->lab2slot;
   int outc = 0;
-  unsigned long long jc = 0;
+  unsigned long long jc = jc0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
                            Oll = (unsigned long long)J.out;
   for (int e0 = 0; e0 < total; e0 += 32) {
@@ -696,6 +708,12 @@ __device__ __forceinline__ void set_sibling(W& w, int F, int u) {
     if (hi < INT_MAX) e = max(b, lbound(p, len, hi));
   }
   if (e - b < lvl_need(w, F, u)) e = b;  // fewer candidates than any extension needs (plan.h need)
+  if (F == 1 && w.kp->entries) {  // a root entry enumerates one piece of its candidate list
+    // (after the need test: the other pattern vertices may come from the whole list)
+    const int c = __ldg(&w.kp->entries[w.h->rent[rsib(w, 1, u)]].y);
+    b = max(b, c * w.kp->root_split);
+    e = max(b, min(e, (c + 1) * w.kp->root_split));
+  }
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->cur[F] = u;
@@ -1091,12 +1109,14 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
 __device__ int gather_roots(W& w) {
   const unsigned rlab = lvl_filt(w, 0, 0).lab;
   const int R = w.kp->root_batch;
+  const int2* ent = w.kp->entries;
   int pos = w.h->root_it;
   const int e = w.h->root_end;
   int m = 0;
   while (m < R && pos < e) {
     const int p = pos + w.lane;
-    const bool pass = p < e && labok(w, p, rlab);
+    const int v = (p < e && ent) ? __ldg(&ent[p].x) : p;
+    const bool pass = p < e && labok(w, v, rlab);
     unsigned pm = __ballot_sync(FULLMASK, pass);
     int room = R - m;
     unsigned acc = pm;
@@ -1107,7 +1127,11 @@ __device__ int gather_roots(W& w) {
       acc = a2;
       cut = true;
     }
-    if ((acc >> w.lane) & 1u) SIB(w, 1, m + __popc(acc & ((1u << w.lane) - 1))) = p;
+    if ((acc >> w.lane) & 1u) {
+      const int slot = m + __popc(acc & ((1u << w.lane) - 1));
+      SIB(w, 1, slot) = v;
+      w.h->rent[slot] = p;
+    }
     m += __popc(acc);
     pos = cut ? pos + (31 - __clz(acc)) + 1 : min(pos + 32, e);
   }
@@ -1381,11 +1405,11 @@ __device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr*
     T.e = v->root_end;
     T.b = v->root_end - s.t;
     v->root_end = T.b;
-  } else if (s.kind == 1) {  // remaining root siblings -> root range
+  } else if (s.kind == 1) {  // remaining root siblings -> root range (entry range)
     const int s0 = v->nsib[1] - s.t;
     T.level = 0;
-    T.b = vsib[1 * STM_RMAX + s0];
-    T.e = vsib[1 * STM_RMAX + v->nsib[1] - 1] + 1;
+    T.b = kp.entries ? v->rent[s0] : vsib[1 * STM_RMAX + s0];
+    T.e = (kp.entries ? v->rent[v->nsib[1] - 1] : vsib[1 * STM_RMAX + v->nsib[1] - 1]) + 1;
     v->nsib[1] = s0;
   } else {
     const int F = s.F;

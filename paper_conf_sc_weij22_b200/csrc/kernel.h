@@ -92,6 +92,12 @@ struct StmKParams {
   int32_t split;                  // 1: narrow rows with the out_start split of vrec (stm_tuning.narrow_split 0)
   const uint32_t* bitmaps;
   int64_t bm_words;
+  // Root entries: when set, the root space [root_lo, n) indexes
+  // entries[] = (root vertex, chunk c) and level 1 of that entry enumerates only positions
+  // [c * root_split, (c + 1) * root_split) of the root's candidate list, so a heavy root is
+  // handed out as several independent pieces from the start.  NULL: root space = vertex ids.
+  const int2* entries;
+  int32_t root_split;
   int64_t n;                      // root space end: roots are [root_lo, n)
   int64_t root_lo;
   int32_t* list_out;              // listing build: [list_cap][k] rows (pattern-vertex order)

@@ -24,6 +24,7 @@
 #define STM_BITMAP_AUTO_MIN_DEGREE 64
 #define STM_BITMAP_AUTO_BUDGET_MB 2048
 #define STM_L2_PERSIST_AUTO_MB 0   // measured neutral at 24-48 MiB, worse at 96 MiB on C5: off
+#define STM_ROOT_SPLIT_AUTO 512    // root splitting piece size (stm_tuning.root_split; measured 32..512 on C2-C5)
 
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
@@ -105,6 +106,12 @@ struct stm_graph {
   std::map<std::tuple<int, int, int64_t>, HubBitmaps> hubs;  // (ranked, min_deg, budget) -> set
   std::mutex mu;
   std::map<void*, Scratch> scratch;  // per stream
+  // root entries per (numbering, piece size) (kernel.h StmKParams::entries), built lazily
+  struct RootEntries {
+    int2* d = nullptr;
+    int64_t n = 0;
+  };
+  std::map<std::pair<int, int>, RootEntries> entries;
   // degree / label statistics of the graph (NEXT-2 cost model), computed at load
   bool has_stats = false;
   stm_graph_stats stats;
@@ -273,6 +280,62 @@ __global__ void hub_fill(int64_t n, int64_t H, const int32_t* rank2orig, const i
       atomicOr(&b[x >> 5], 1u << (x & 31));
     }
   }
+}
+
+// ---------------------------------------------------------------- root entries
+__global__ void entry_counts(const int64_t* rp, int64_t n, int T, int64_t* cnt) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t d = rp[v + 1] - rp[v];
+    cnt[v] = d > T ? (d + T - 1) / T : 1;
+  }
+}
+__global__ void entry_fill(const int64_t* off, int64_t n, int2* out) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    for (int64_t c = 0; c < off[v + 1] - off[v]; ++c) out[off[v] + c] = make_int2((int)v, (int)c);
+}
+
+// Entries (v, piece) in vertex order for the numbering `ranked`; caller holds g->mu.
+// NULL (no splitting) on any failure -- speed only.
+static const stm_graph::RootEntries* ensure_entries(stm_graph* g, bool ranked, int T) {
+  const auto key = std::make_pair(ranked ? 1 : 0, T);
+  auto it = g->entries.find(key);
+  if (it != g->entries.end()) return it->second.d ? &it->second : nullptr;
+  stm_graph::RootEntries& E = g->entries[key];
+  const int64_t n = g->n;
+  if (n < 1 || T < 1) return nullptr;
+  const int64_t* rp = ranked ? g->d_rrow_ptr : g->d_row_ptr;
+  int64_t* off = nullptr;
+  void* temp = nullptr;
+  size_t tb = 0;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 4096);
+  cudaError_t e = cudaMalloc(&off, sizeof(int64_t) * (n + 1));
+  if (e == cudaSuccess) {
+    entry_counts<<<grid, 256>>>(rp, n, T, off);
+    e = cudaMemset(off + n, 0, sizeof(int64_t));
+  }
+  if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, off, off, (int)(n + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&temp, std::max<size_t>(tb, 16));
+  if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(temp, tb, off, off, (int)(n + 1));
+  int64_t total = 0;
+  if (e == cudaSuccess) e = cudaMemcpy(&total, off + n, sizeof total, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && total < INT32_MAX) {
+    e = cudaMalloc(&E.d, sizeof(int2) * (size_t)total);
+    if (e == cudaSuccess) {
+      entry_fill<<<grid, 256>>>(off, n, E.d);
+      e = cudaGetLastError();
+      if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    }
+  }
+  cudaFree(off);
+  cudaFree(temp);
+  if (e != cudaSuccess || total >= INT32_MAX || !E.d) {
+    cudaGetLastError();
+    cudaFree(E.d);
+    E.d = nullptr;
+    return nullptr;
+  }
+  E.n = total;
+  return &E;
 }
 
 static void free_hub(stm_graph::HubBitmaps& h) {
@@ -565,6 +628,7 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
   cudaFree(g->d_out_start);
   cudaFree(g->d_rout_start);
   for (auto& kv : g->hubs) free_hub(kv.second);
+  for (auto& kv : g->entries) cudaFree(kv.second.d);
   delete g;
   return STM_OK;
 }
@@ -620,6 +684,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.watchdog_ms < 0) return stm_fail(STM_EINVAL, "watchdog_ms %d < 0", t.watchdog_ms);
   if (t.backoff_max < 0 || t.backoff_max > 12) return stm_fail(STM_EINVAL, "backoff_max %d not in 0..12", t.backoff_max);
   if (t.carveout_pct < -1 || t.carveout_pct > 100) return stm_fail(STM_EINVAL, "carveout_pct %d", t.carveout_pct);
+  if (t.root_split < -1) return stm_fail(STM_EINVAL, "root_split %d", t.root_split);
   if (d_result && ((uintptr_t)d_result & 7)) return stm_fail(STM_EINVAL, "d_result not 8-byte aligned");
   const StmPlan& P = p->dev;
   if (!p->labels.empty() && !g->d_labels) {
@@ -660,6 +725,16 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     kp.bitmaps = hb->bits;
     kp.bm_words = hb->words;
     g_info.hubs = hb->n_hubs;
+    // root splitting (stm_tuning.root_split): not for listing pages, which are root-id ranges
+    const int T = t.root_split == 0 ? STM_ROOT_SPLIT_AUTO : t.root_split;
+    if (!la && T > 0) {
+      const stm_graph::RootEntries* E = ensure_entries(g, use_rank, T);
+      if (E) {
+        kp.entries = E->d;
+        kp.root_split = T;
+        kp.n = E->n;
+      }
+    }
   }
   // label-slot table: dense graph label -> bitmask of pattern slots with that value
   for (int d = 0; d < (int)g->label_values.size(); ++d)

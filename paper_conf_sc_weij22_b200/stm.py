@@ -43,7 +43,7 @@ class stm_tuning(ctypes.Structure):
                                                "instrument", "hash_slots", "vertex_order",
                                                "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
                                                "l2_persist_mb", "drive_ratio", "narrow_split", "watchdog_ms",
-                                               "backoff_max", "carveout_pct")]
+                                               "backoff_max", "carveout_pct", "root_split")]
 
 
 class stm_shard(ctypes.Structure):

@@ -128,6 +128,9 @@ TUNINGS = [
     dict(occupancy=2, unroll=5, root_chunk=1, stop_level=3, detect_level=3),
     dict(root_order=1), dict(root_order=2, vertex_order=1), dict(root_order=2, root_chunk=3, occupancy=2),
     dict(l2_persist_mb=8, occupancy=2),
+    dict(root_split=-1), dict(root_split=1), dict(root_split=3, root_chunk=5, stop_level=3),
+    dict(root_split=2, vertex_order=1, root_order=2), dict(root_split=4, root_chunk=1, unroll=2),
+    dict(backoff_max=1, carveout_pct=-1), dict(backoff_max=12, carveout_pct=50),
 ]
 
 
