@@ -144,10 +144,14 @@ stm_status stm_plan_free(stm_plan* p);
 
 /* Tuning knobs: every setting changes speed only, never the count. NULL = defaults. */
 typedef struct stm_tuning {
-  int32_t local_steal;    /* 0/1: intra-block stealing through shared memory (Sec. V-A). Default 1. */
-  int32_t global_steal;   /* 0/1: inter-block stealing through global mailboxes (Sec. V-B). Default 1. */
-  int32_t stop_level;     /* frames < stop_level are stealable (paper: 2). Default 2. */
-  int32_t detect_level;   /* donors look for idle blocks at frames < detect_level (paper: 1). Default 2. */
+  int32_t local_steal;    /* 0/1: intra-block work sharing through shared-memory mailboxes (Sec. V-A,
+                             re-designed: busy warps split their own stacks on request).  Default 1. */
+  int32_t global_steal;   /* 0/1: inter-block work sharing through a grid-wide task pool (Sec. V-B,
+                             re-designed: DESIGN.md "Stealing").  Default 1. */
+  int32_t stop_level;     /* frames < stop_level are donated (paper: 2); while more than
+                             1/8 of the warps are idle every frame is.  Default 2. */
+  int32_t detect_level;   /* donors look at the grid-wide pool's demand at frames < detect_level (paper:
+                             idle blocks, 1).  Default 8 (every frame). */
   int32_t unroll;         /* sibling iterations expanded together, 1..32 (paper: 8);
                              0 = auto (32 with the 40-register kernel, else 16; measured).  Default 0. */
   int32_t root_chunk;     /* roots per cursor grab, 1..32; 0 = auto (1 with the 64-register kernel,
@@ -200,6 +204,13 @@ typedef struct stm_tuning {
                              (c+1)*root_split) of its level-1 candidate list, so the heaviest roots are
                              spread over many warps from the start instead of being split by stealing.
                              0 = auto (512), -1 = off (one piece per root).  Speed only. */
+  int32_t chunk_cost;     /* work-balanced root chunks: consecutive root entries are grouped into one
+                             cursor chunk until their estimated cost (1 + candidate-list length each)
+                             reaches chunk_cost, so the light bulk of a power-law graph is handed out
+                             many roots per atomic and every heavy root (piece) alone.  0 = auto
+                             (min(512, (n + nnz) / (8 * 48 * SMs)), at least 16: ~8 chunks per warp),
+                             -1 = off (fixed root_chunk roots per chunk).  Counting launches only (not
+                             listing pages).  Speed only. */
 } stm_tuning;
 
 /* Fill t with the defaults. */

@@ -116,17 +116,33 @@
     atomicAdd(pl + 1, 1ull);                                                                        \
     atomicAdd(pl + 2, (unsigned long long)w.last_total);                                            \
   }
+// longest busy interval between two work-sharing checks: the indivisible unit of work
+// (the critical path a split can never shorten)
+#define PROF_CHK()                                                                      \
+  if (w.lane == 0) {                                                                    \
+    const long long now_ = clock64();                                                   \
+    if (w.prof_chk)                                                                     \
+      atomicMax(&w.kp->work->prof[3 * STM_PROF_N + 4 + STM_PROF_LVL - 2],               \
+                (unsigned long long)(now_ - w.prof_chk));                               \
+    w.prof_chk = now_;                                                                  \
+    prof_timeline(w);                                                                   \
+  }
 #else
 #define PROF_BEGIN(id)
 #define PROF_END(id, items)
 #define PROF_LVL_BEGIN()
 #define PROF_LVL_END(kind, lvl)
+#define PROF_CHK()
 #endif
 
 namespace {
 
 struct WarpHdr {
-  int lock;
+  // Local work sharing: an idle warp sets its bit in
+  // BlockHdr::idle_mask and waits; a busy warp of the block that sees the bit claims
+  // it (clears it with an atomic), splits its OWN stack and posts the task here.  Only
+  // the owner ever reads or writes a stack, so the busy path takes no locks.
+  int mail_full;              // 1 when `mail` holds a task donated to this warp
   int L;                      // current frame (0 = root level)
   int root_it, root_end;      // frame 0: remaining root-ID range of the current chunk
   int nsib[STM_KMAX], cur[STM_KMAX], it[STM_KMAX], end[STM_KMAX];
@@ -139,17 +155,22 @@ struct WarpHdr {
   int steal_fails;
   int pad0;
   long long first_dry;        // STM_PROFILE: clock64() when the root cursors were first seen exhausted
+  long long gchk;             // clock64() of the last look at the pool's demand
+  long long wd0;              // %globaltimer at the warp's start (watchdog)
+  int deep;                   // 1: donate from every frame (grid starving, split_stop)
+  int pad1;
   // STM_MULTI: frame F iterates the virtual siblings vs = child * nr[F] + u, u < nr[F]
   // the real sibling (value of v_{F-1}) and child the child of trie vertex pv[F] whose
   // candidates are enumerated (child-major: consecutive virtual siblings share a child,
   // so the last level's counts pack up to 32 (sibling, candidate) pairs of one child)
   int pv[STM_KMAX], nr[STM_KMAX];
   int rent[STM_RMAX];         // root entries (kp.entries): entry index of frame-1 sibling u
+  StmTask mail;               // the donated task (valid while mail_full == 1)
 };
 
 struct BlockHdr {
-  int idle_mask;
-  int leader;
+  int idle_mask;              // warps idle and waiting for a donation (bit per warp)
+  int poller;                 // the idle warp that polls the grid-wide pool (-1: none)
   int done;
   int pad;
   unsigned char lab2slot[256];
@@ -182,6 +203,10 @@ struct W {
 #if STM_PROFILE
   unsigned long long prof_cyc[STM_PROF_N], prof_cnt[STM_PROF_N], prof_items[STM_PROF_N];
   int last_total;  // elements driven by the last combined operation
+  long long prof_chk;  // clock64() of the last work-sharing check (0: idle since)
+  long long prof_g;    // %globaltimer of the last check (0: idle since)
+  int prof_b;          // timeline bucket being accumulated in prof_acc
+  unsigned long long prof_acc;
 #endif
 };
 
@@ -208,9 +233,42 @@ __device__ __forceinline__ W make_w(const StmKParams& kp) {
   w.idle_cyc = 0;
 #if STM_PROFILE
   for (int i = 0; i < STM_PROF_N; ++i) w.prof_cyc[i] = w.prof_cnt[i] = w.prof_items[i] = 0;
+  w.prof_chk = 0;
+  w.prof_g = 0;
+  w.prof_b = 0;
+  w.prof_acc = 0;
 #endif
   return w;
 }
+
+#if STM_PROFILE
+// busy time since the last check, credited to the timeline bucket of now (lane 0)
+__device__ __forceinline__ void prof_timeline(W& w) {
+  long long g;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+  if (w.prof_g) {
+    const int b = (int)((g - w.h->wd0) / STM_PROF_TL_NS);
+    if (b != w.prof_b) {
+      if (w.prof_acc && w.prof_b >= 0 && w.prof_b < STM_PROF_TL)
+        atomicAdd(&w.kp->work->prof[3 * STM_PROF_N + 4 + STM_PROF_LVL + w.prof_b], w.prof_acc);
+      w.prof_acc = 0;
+      w.prof_b = b;
+    }
+    w.prof_acc += (unsigned long long)(g - w.prof_g);
+  }
+  w.prof_g = g;
+}
+__device__ __forceinline__ void prof_timeline_flush(W& w) {
+  if (w.lane == 0 && w.prof_acc && w.prof_b >= 0 && w.prof_b < STM_PROF_TL)
+    atomicAdd(&w.kp->work->prof[3 * STM_PROF_N + 4 + STM_PROF_LVL + w.prof_b], w.prof_acc);
+  w.prof_acc = 0;
+}
+#endif
+
+// donor sides of local / global work sharing (defined with the scheduler below)
+__device__ __noinline__ void share_local(const StmKParams& kp);
+__device__ __noinline__ void maybe_push(const StmKParams& kp);
+__device__ __noinline__ bool watchdog(const StmKParams& kp, long long t0, const char* where);
 
 // instrumented builds: add a W's per-lane algorithmic-byte partials to the launch totals
 __device__ __forceinline__ void flush_instr(W& w) {
@@ -658,28 +716,28 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
 #endif
 
 // ----------------------------------------------------------------------------
-// locks and small helpers
+// small helpers
 // ----------------------------------------------------------------------------
-__device__ __forceinline__ void lock_ws(const W& w, volatile WarpHdr* h) {
+// warps of this block waiting for a donation (uniform across the warp)
+__device__ __forceinline__ int waiting_warps(const W& w) {
+  int m = 0;
+  if (w.lane == 0) m = *(volatile int*)&w.bh->idle_mask;
+  return __shfl_sync(FULLMASK, m, 0);
+}
+// Grid status, looked at (two L2 loads) at most every ~0.5 us per warp: does the pool want
+// a task (block pollers waiting)?  Is the grid starving (WarpHdr::deep, split_stop)?
+__device__ __forceinline__ bool pool_wanted(const W& w) {
+  int want = 0;
   if (w.lane == 0) {
-    while (atomicCAS((int*)&h->lock, 0, 1) != 0) __nanosleep(32);
-    __threadfence_block();
+    const long long now = clock64();
+    if (now - w.h->gchk >= 1024) {
+      w.h->gchk = now;
+      volatile StmWork* vw = w.kp->work;
+      want = vw->deficit > 0;
+      w.h->deep = 8 * (w.kp->total_warps - vw->active) > w.kp->total_warps;
+    }
   }
-  __syncwarp();
-}
-__device__ __forceinline__ void unlock_ws(const W& w, volatile WarpHdr* h) {
-  __syncwarp();
-  if (w.lane == 0) {
-    __threadfence_block();
-    atomicExch((int*)&h->lock, 0);
-  }
-  __syncwarp();
-}
-__device__ __forceinline__ bool stealing(const W& w) {
-  return w.kp->local_steal || w.kp->global_steal;
-}
-__device__ __forceinline__ bool locked_frame(const W& w, int F) {
-  return stealing(w) && F < w.kp->stop_level;
+  return __shfl_sync(FULLMASK, want, 0) != 0;
 }
 
 // candidate-list length of frame F's sibling u
@@ -1174,9 +1232,13 @@ __device__ void frame_count(W& w, int m) {
 #if !STM_MULTI
 __device__ STEP_INL void fused_count(W& w, int F) {
   const StmPlan& P = *w.P;
-  const bool lk = locked_frame(w, F);
-  for (;;) {
-    if (lk) lock_ws(w, w.h);
+  for (unsigned pass = 1;; ++pass) {
+    if ((pass & 63) == 0 && watchdog(*w.kp, w.h->wd0, "fused")) return;  // (the main loop aborts next)
+    // share with waiting warps of the block between counting passes (the stack is
+    // consistent here: the staged pairs were already taken out of [it, end))
+    PROF_CHK()
+    if (w.kp->local_steal && waiting_warps(w)) share_local(*w.kp);
+    if (pool_wanted(w) && w.kp->global_steal && F < w.kp->detect_level) maybe_push(*w.kp);
     int nj = 0;
     // gather up to 32 passing candidates across siblings
     for (;;) {
@@ -1224,7 +1286,6 @@ __device__ STEP_INL void fused_count(W& w, int F) {
       __syncwarp();
       if (nj == 32) break;
     }
-    if (lk) unlock_ws(w, w.h);
     if (nj == 0) return;
     Job J;
     J.A = nullptr; J.B = nullptr; J.alen = 0; J.blen = 0; J.op = STM_OP_NONE;
@@ -1244,9 +1305,10 @@ __device__ STEP_INL void fused_count(W& w, int F) {
 // child-major) and count every leaf below it over them.  Returns when the frame is
 // exhausted or reaches a child that needs level-(k-1) sets (the frame path builds those).
 __device__ STEP_INL void fused_count_multi(W& w, int F) {
-  const bool lk = locked_frame(w, F);
-  for (;;) {
-    if (lk) lock_ws(w, w.h);
+  for (unsigned pass = 1;; ++pass) {
+    if ((pass & 63) == 0 && watchdog(*w.kp, w.h->wd0, "fused")) return;  // (the main loop aborts next)
+    if (w.kp->local_steal && waiting_warps(w)) share_local(*w.kp);
+    if (pool_wanted(w) && w.kp->global_steal && F < w.kp->detect_level) maybe_push(*w.kp);
     int nj = 0, child = -1;
     for (;;) {
       const int u = w.h->cur[F];
@@ -1296,7 +1358,6 @@ __device__ STEP_INL void fused_count_multi(W& w, int F) {
       __syncwarp();
       if (nj == 32) break;
     }
-    if (lk) unlock_ws(w, w.h);
     if (nj == 0) return;
     const StmMVert& sv = mvert(w, child);
     for (int lv = sv.child_begin; lv < sv.child_begin + sv.n_children; ++lv) {
@@ -1326,6 +1387,17 @@ __device__ __noinline__ bool try_chunk(const StmKParams& kp) {
       if (!kp.cursors[r] || (ex & (1u << r))) continue;
       unsigned long long idx = atomicAdd(kp.cursors[r], 1ull);
       long long c = (long long)r + (long long)kp.world * (long long)idx;
+      if (kp.chunk_bounds) {  // work-balanced chunks (positions [bounds[c], bounds[c+1]))
+        if (c < kp.n_chunks) {
+          if (kp.root_desc) c = kp.n_chunks - 1 - c;  // the heaviest (last) chunks first
+          from = r;
+          b = __ldg(&kp.chunk_bounds[c]);
+          e = __ldg(&kp.chunk_bounds[c + 1]);
+        } else {
+          ex |= 1u << r;
+        }
+        continue;
+      }
       long long rb = kp.root_lo + c * (long long)kp.chunk;
       if (rb < kp.n) {
         from = r;
@@ -1348,14 +1420,13 @@ __device__ __noinline__ bool try_chunk(const StmKParams& kp) {
   b = bcast(b);
   e = bcast(e);
   if (b < 0) return false;
-  lock_ws(w, w.h);
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) {
     w.h->root_it = b;
     w.h->root_end = e;
     w.h->L = 0;
   }
-  unlock_ws(w, w.h);
+  __syncwarp();
   if (w.lane == 0) {
     atomicAdd(&kp.work->n_chunks, 1ull);
     if (from != kp.rank) atomicAdd(&kp.work->n_peer_chunks, 1ull);
@@ -1363,16 +1434,26 @@ __device__ __noinline__ bool try_chunk(const StmKParams& kp) {
   return true;
 }
 
-// What a steal from stack `v` would take (half of the
-// shallowest stealable remaining work).  Work at the victim's current frame L is
-// not in progress yet, so there the victim always keeps at least one item
-// (otherwise a single item could be passed around forever); at frames shallower
-// than L the victim is busy below and the thief may take it all.
-// kind: 0 = root range of frame 0, 1 = remaining root siblings of frame 1,
-// 2 = remaining candidates of the current sibling of frame F.  F < 0: nothing.
+// What a donation from the warp's own stack `v` gives away (the
+// shallowest stealable remaining work).  Work at the donor's current frame L is not in
+// progress yet, so there the donor always keeps at least one item (otherwise a single
+// item could be passed around forever); at frames shallower than L the donor is busy
+// below and may give it all.
+// kind: 0 = half the root range of frame 0, 1 = half the remaining root siblings of
+// frame 1, 2 = half the remaining candidates of the current sibling of frame F,
+// 3 = the last not-yet-started sibling of frame F >= 2, whole.  F < 0: nothing.
 struct SplitPick {
   int F, kind, t;
 };
+
+// Depth limit of donations: frames < stop_level normally; every frame while the grid is
+// starving (more than 1/8 of the warps idle, WarpHdr::deep refreshed by grid_status).
+// Deep donations make the receiver rebuild the donor's prefix sets, which costs as much
+// as the donor's own builds (K6-e: the hub-pair intersections), so they are kept for the
+// tail, where idle warps would otherwise wait.
+__device__ __forceinline__ int split_stop(const StmKParams& kp, volatile WarpHdr* v) {
+  return v->deep ? STM_KMAX : kp.stop_level;
+}
 
 __device__ __forceinline__ SplitPick pick_split(int stop, volatile WarpHdr* v) {
   const int L = v->L;
@@ -1383,10 +1464,12 @@ __device__ __forceinline__ SplitPick pick_split(int stop, volatile WarpHdr* v) {
     const int cur = v->cur[F], nsib = v->nsib[F];
     if (cur >= nsib) continue;
     const int rem = v->end[F] - v->it[F];
+    const int rs = nsib - cur - 1;  // siblings not started yet
     if (F == 1 && !STM_MULTI) {  // (merged plans: child-major frames have no whole-sibling split)
-      const int rs = nsib - cur - 1;
       const int ts = (L > 1 || rem > 0) ? (rs + 1) / 2 : rs / 2;
       if (ts >= 1) return {1, 1, ts};
+    } else if (!STM_MULTI && rs >= 1) {
+      return {F, 3, 1};
     }
     const bool last_sib = cur + 1 >= nsib;
     const int tr = (L > F || !last_sib) ? (rem + 1) / 2 : rem / 2;
@@ -1395,10 +1478,10 @@ __device__ __forceinline__ SplitPick pick_split(int stop, volatile WarpHdr* v) {
   return {-1, 0, 0};
 }
 
-// Split the stack of `v` (caller holds v's lock).  Returns false if nothing.
+// Split the warp's own stack `v` (only its owner calls this).  Returns false if nothing.
 __device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr* v, volatile int* vsib,
                                         StmTask& T) {
-  const SplitPick s = pick_split(kp.stop_level, v);
+  const SplitPick s = pick_split(split_stop(kp, v), v);
   if (s.F < 0) return false;
   if (s.kind == 0) {
     T.level = 0;
@@ -1411,6 +1494,15 @@ __device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr*
     T.b = kp.entries ? v->rent[s0] : vsib[1 * STM_RMAX + s0];
     T.e = (kp.entries ? v->rent[v->nsib[1] - 1] : vsib[1 * STM_RMAX + v->nsib[1] - 1]) + 1;
     v->nsib[1] = s0;
+  } else if (s.kind == 3) {  // the last unstarted sibling u of frame F: prefix v_0..v_{F-2}, v_{F-1} = SIB(F, u)
+    const int F = s.F;
+    const int u = v->nsib[F] - 1;
+    T.level = F;
+    T.b = -1;  // its whole (bound-narrowed) candidate list: the receiver runs set_sibling
+    T.e = -1;
+    for (int j = 0; j < F - 1; ++j) T.prefix[j] = vsib[(j + 1) * STM_RMAX + v->cur[j + 1]];
+    T.prefix[F - 1] = vsib[F * STM_RMAX + u];
+    v->nsib[F] = u;
   } else {
     const int F = s.F;
     T.level = F;
@@ -1428,16 +1520,6 @@ __device__ __noinline__ bool split_stack(const StmKParams& kp, volatile WarpHdr*
   return true;
 }
 
-// amount-of-work score of a stack (higher = better victim; 0 = nothing a split
-// would take), racy read without the lock
-__device__ __forceinline__ int steal_score(int stop, volatile WarpHdr* v) {
-  const SplitPick s = pick_split(stop, v);
-  if (s.F < 0) return 0;
-  if (s.F == 0) return 1 << 30;
-  return ((STM_KMAX - s.F) << 24) + min(s.t * (s.kind == 1 ? 1024 : 1), (1 << 24) - 1);
-}
-
-
 __device__ __forceinline__ long long gtimer() {
   long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -1448,16 +1530,18 @@ __device__ __forceinline__ long long gtimer() {
 // than watchdog_ns of wall time; the launch then aborts and reports STM_ETIMEOUT
 // (work->overflow = 2), never a partial count.  STM_DEBUG builds also dump state.
 __device__ __noinline__ bool watchdog(const StmKParams& kp, long long t0, const char* where) {
-  if (!kp.watchdog_ns || gtimer() - t0 < kp.watchdog_ns) return false;
+  if (!kp.watchdog_ns) return false;
+  // once one warp has fired, every warp aborts at its next check
+  if (*(volatile int*)&kp.work->overflow != 2 && gtimer() - t0 < kp.watchdog_ns) return false;
   W w = make_w(kp);
   if (w.lane == 0) {
     atomicExch(&w.kp->work->overflow, 2);
 #if STM_DEBUG
     volatile WarpHdr* h = w.h;
-    printf("WATCHDOG %s blk %d warp %d L=%d root=[%d,%d) nsib1=%d cur1=%d it1=%d end1=%d idle_blocks=%d mask=%x leader=%d is_idle=%d mail=%d\n",
+    printf("WATCHDOG %s blk %d warp %d L=%d root=[%d,%d) nsib1=%d cur1=%d it1=%d end1=%d active=%d started=%d deficit=%d mask=%x poller=%d mail=%d\n",
            where, blockIdx.x, w.wid, h->L, h->root_it, h->root_end, h->nsib[1], h->cur[1], h->it[1], h->end[1],
-           *(volatile int*)&w.kp->work->idle_blocks, w.bh->idle_mask, w.bh->leader,
-           w.kp->slots[blockIdx.x].is_idle, w.kp->slots[blockIdx.x].mail_full);
+           *(volatile int*)&w.kp->work->active, *(volatile int*)&w.kp->work->started,
+           *(volatile int*)&w.kp->work->deficit, w.bh->idle_mask, w.bh->poller, h->mail_full);
 #else
     (void)where;
 #endif
@@ -1470,16 +1554,14 @@ __device__ __noinline__ bool watchdog(const StmKParams& kp, long long t0, const 
 // levels 1..T.level from the prefix).
 __device__ __noinline__ void adopt_task(const StmKParams& kp, const StmTask& T) {
   W w = make_w(kp);
-  const int k = w.P->k;
   if (T.level == 0) {
-    lock_ws(w, w.h);
     HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
       w.h->root_it = T.b;
       w.h->root_end = T.e;
       w.h->L = 0;
     }
-    unlock_ws(w, w.h);
+    __syncwarp();
     return;
   }
   const int l = T.level;
@@ -1510,19 +1592,22 @@ __device__ __noinline__ void adopt_task(const StmKParams& kp, const StmTask& T) 
       __syncwarp();
       build_nodes(w, i - 1, 1, false);  // a stolen prefix is rebuilt as given
     }
-    int len = src_len(w, i, w.h->cur[i]);
-    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-    if (w.lane == 0) {
-      w.h->it[i] = (i == l) ? T.b : len;
-      w.h->end[i] = (i == l) ? min(T.e, len) : len;
+    if (i == l && T.b < 0) {
+      // a whole sibling (split kind 3): its bound-narrowed candidate range
+      set_sibling(w, i, w.h->cur[i]);
+    } else {
+      const int len = src_len(w, i, w.h->cur[i]);
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+      if (w.lane == 0) {
+        w.h->it[i] = (i == l) ? T.b : len;
+        w.h->end[i] = (i == l) ? min(T.e, len) : len;
+      }
+      __syncwarp();
     }
-    __syncwarp();
   }
-  (void)k;
-  lock_ws(w, w.h);
   HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
   if (w.lane == 0) w.h->L = l;
-  unlock_ws(w, w.h);
+  __syncwarp();
   flush_instr(w);  // the rebuild's set operations count toward W
 }
 
@@ -1530,35 +1615,26 @@ __device__ __forceinline__ volatile WarpHdr* warp_hdr(const W& w, int wid) {
   const int wb = warp_bytes(w.P->k, w.P->n_nodes, w.kp->ht_slots);
   return (volatile WarpHdr*)(stm_smem + sizeof(BlockHdr) + (size_t)wid * wb);
 }
-__device__ __forceinline__ volatile int* warp_sib(const W& w, int wid) {
-  return (volatile int*)((volatile unsigned char*)warp_hdr(w, wid) + sizeof(WarpHdr));
-}
 
-__device__ __noinline__ bool try_local_steal(const StmKParams& kp) {
-  W w = make_w(kp);
-  const int nw = kp.block_warps;
-  // pick the best victim (racy scores), then split under its lock
-  int best = -1, bs = 0;
-  if (w.lane < nw && w.lane != w.wid) {
-    int s = steal_score(kp.stop_level, warp_hdr(w, w.lane));
-    if (s > 0) { best = w.lane; bs = s; }
+__device__ __forceinline__ void write_task(volatile StmTask* M, const StmTask& T) {
+  M->level = T.level;
+  M->b = T.b;
+  M->e = T.e;
+  for (int j = 0; j < STM_KMAX; ++j) {
+    M->prefix[j] = T.prefix[j];
+    M->tv[j] = T.tv[j];
   }
-  // warp argmax (lowest id on ties)
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    int ob = __shfl_xor_sync(FULLMASK, best, o);
-    int os = __shfl_xor_sync(FULLMASK, bs, o);
-    if (os > bs || (os == bs && ob >= 0 && (best < 0 || ob < best))) { best = ob; bs = os; }
+}
+__device__ __forceinline__ void read_task(volatile StmTask* M, StmTask& T) {
+  T.level = M->level;
+  T.b = M->b;
+  T.e = M->e;
+  for (int j = 0; j < STM_KMAX; ++j) {
+    T.prefix[j] = M->prefix[j];
+    T.tv[j] = M->tv[j];
   }
-  if (best < 0) return false;
-  volatile WarpHdr* v = warp_hdr(w, best);
-  StmTask T;
-  int ok = 0;
-  lock_ws(w, v);
-  if (w.lane == 0) ok = split_stack(kp, v, warp_sib(w, best), T);
-  unlock_ws(w, v);
-  ok = bcast(ok);
-  if (!ok) return false;
+}
+__device__ __forceinline__ void bcast_task(StmTask& T) {
   T.level = bcast(T.level);
   T.b = bcast(T.b);
   T.e = bcast(T.e);
@@ -1566,174 +1642,172 @@ __device__ __noinline__ bool try_local_steal(const StmKParams& kp) {
     T.prefix[j] = bcast(T.prefix[j]);
     T.tv[j] = (int16_t)bcast(T.tv[j]);
   }
-  if (w.lane == 0) atomicAdd(&kp.work->n_local_steals, 1ull);
-  adopt_task(kp, T);
-  return true;
 }
 
-// donor side of Fig. 6: give half of my shallowest work to an idle block
-__device__ __noinline__ void maybe_donate(const StmKParams& kp) {
+// Donor side of local work sharing (Sec. V-A, re-designed: the busy
+// warp splits its own stack instead of an idle warp splitting it under a lock).
+// Called by a busy warp that saw waiting warps in its block: claim one (clear its
+// idle bit), give it the shallowest stealable part of this stack.
+__device__ __noinline__ void share_local(const StmKParams& kp) {
   W w = make_w(kp);
-  // the idle-block count lives in L2: look at it on every (donate_mask+1)-th opportunity
-  unsigned tick = 0;
-  if (w.lane == 0) tick = ++w.h->donate_tick;
-  tick = __shfl_sync(FULLMASK, tick, 0);
-  if ((tick & (unsigned)kp.donate_mask) != 0) return;
-  int idle = 0;
-  if (w.lane == 0) idle = *(volatile int*)&kp.work->idle_blocks;
-  idle = bcast(idle);
-  if (idle <= 0) return;
-  // only donate what a split can actually take
-  if (pick_split(kp.stop_level, w.h).F < 0) return;
-  const int nb = gridDim.x;
-  int target = -1;
-  const int off = (int)((blockIdx.x * 37u + w.wid * 11u + tick) % (unsigned)nb);
-  for (int b0 = 0; b0 < min(nb, 64) && target < 0; b0 += 32) {
-    int b = (off + b0 + w.lane) % nb;
-    bool cand = (b0 + w.lane < nb) && b != (int)blockIdx.x &&
-                *(volatile int*)&kp.slots[b].is_idle == 1;
-    unsigned cm = __ballot_sync(FULLMASK, cand);
-    while (cm && target < 0) {
-      int l = __ffs(cm) - 1;
-      cm &= cm - 1;
-      int tb = __shfl_sync(FULLMASK, b, l);
-      int got = 0;
-      if (w.lane == 0) got = atomicCAS(&kp.slots[tb].is_idle, 1, 2) == 1;
-      if (bcast(got)) target = tb;
+  if (w.lane == 0 && pick_split(split_stop(kp, w.h), w.h).F >= 0) {
+    unsigned want = (unsigned)*(volatile int*)&w.bh->idle_mask & ~(1u << w.wid);
+    int target = -1;
+    while (want && target < 0) {
+      const int t = __ffs(want) - 1;
+      want &= want - 1;
+      if ((atomicAnd(&w.bh->idle_mask, ~(1 << t)) >> t) & 1) target = t;
     }
-  }
-  if (target < 0) return;
-  StmTask T;
-  int ok = 0;
-  lock_ws(w, w.h);
-  if (w.lane == 0) ok = split_stack(kp, w.h, w.sib, T);
-  unlock_ws(w, w.h);
-  if (w.lane == 0) {
-    if (!ok) {
-      atomicExch(&kp.slots[target].is_idle, 1);
-    } else {
-      volatile StmTask* M = &kp.slots[target].mail;
-      M->level = T.level;
-      M->b = T.b;
-      M->e = T.e;
+    if (target >= 0) {
+      atomicAdd(&kp.work->active, 1);  // the claimed warp is busy from now on (termination)
+      StmTask T;
       for (int j = 0; j < STM_KMAX; ++j) {
-        M->prefix[j] = T.prefix[j];
-        M->tv[j] = T.tv[j];
+        T.prefix[j] = 0;
+        T.tv[j] = 0;
       }
-      __threadfence();
-      atomicSub(&kp.work->idle_blocks, 1);
-      __threadfence();
-      atomicExch(&kp.slots[target].mail_full, 1);
-      atomicAdd(&kp.work->n_global_steals, 1ull);
+      split_stack(kp, w.h, w.sib, T);  // succeeds: only this warp changes its own stack
+      volatile WarpHdr* th = warp_hdr(w, target);
+      write_task(&th->mail, T);
+      __threadfence_block();
+      th->mail_full = 1;
+      atomicAdd(&kp.work->n_local_steals, 1ull);
     }
   }
   __syncwarp();
 }
 
+// Donor side of global work sharing (Sec. V-B, re-designed for B200:
+// a grid-wide task pool instead of per-block mailboxes).  Busy warps look at the pool's
+// deficit (block pollers waiting minus queued tasks); a donor that claims one unit of it
+// splits its own stack and queues the shallowest stealable part.
+__device__ __noinline__ void maybe_push(const StmKParams& kp) {
+  W w = make_w(kp);
+  if (w.lane == 0 && *(volatile int*)&kp.work->deficit > 0 && pick_split(split_stop(kp, w.h), w.h).F >= 0) {
+    if (atomicSub(&kp.work->deficit, 1) > 0) {
+      StmTask T;
+      for (int j = 0; j < STM_KMAX; ++j) {
+        T.prefix[j] = 0;
+        T.tv[j] = 0;
+      }
+      split_stack(kp, w.h, w.sib, T);    // succeeds: only this warp changes its own stack
+      atomicAdd(&kp.work->active, 1);    // the queued task keeps the launch alive
+      const unsigned long long t = atomicAdd(&kp.work->pool_tail, 1ull);
+      StmPoolSlot* s = &kp.pool[t & (unsigned long long)kp.pool_mask];
+      const int free_seq = (int)(2ull * (t >> kp.pool_shift));
+      while (*(volatile int*)&s->seq != free_seq) __nanosleep(64);  // (the pool never fills: deficit)
+      write_task(&s->task, T);
+      __threadfence();
+      atomicExch(&s->seq, free_seq + 1);
+      atomicAdd(&kp.work->n_global_steals, 1ull);
+    } else {
+      atomicAdd(&kp.work->deficit, 1);
+    }
+  }
+  __syncwarp();
+}
+
+// Pop one task from the pool (lane 0).  Returns false if the pool looked empty.
+__device__ __forceinline__ bool pool_pop(const StmKParams& kp, StmTask& T) {
+  volatile StmWork* vw = kp.work;
+  for (;;) {
+    const unsigned long long h = vw->pool_head, t = vw->pool_tail;
+    if (h >= t) return false;
+    if (atomicCAS(&kp.work->pool_head, h, h + 1) != h) continue;
+    StmPoolSlot* s = &kp.pool[h & (unsigned long long)kp.pool_mask];
+    const int full_seq = (int)(2ull * (h >> kp.pool_shift)) + 1;
+    while (*(volatile int*)&s->seq != full_seq) __nanosleep(32);  // the pusher is writing it
+    __threadfence();
+    read_task(&s->task, T);
+    atomicExch(&s->seq, full_seq + 1);  // free for the next round
+    return true;
+  }
+}
+
 // No more local work: returns true with new work adopted, false on termination.
+// The warp leaves the active set and sets its bit in the block's idle mask (a busy warp
+// of the block may then claim it and post a task into its mailbox).  One idle warp per
+// block -- the poller -- also pops tasks from the grid-wide pool and detects termination:
+// every warp started and `active` == 0 (no busy warp, no queued or claimed task).
 __device__ __noinline__ bool acquire_work(const StmKParams& kp, long long t0) {
   W w = make_w(kp);
   if (try_chunk(kp)) return true;
   if (!kp.local_steal && !kp.global_steal) return false;
-  if (kp.local_steal && try_local_steal(kp)) return true;
   BlockHdr* bh = w.bh;
-  const unsigned all = (kp.block_warps == 32) ? FULLMASK : ((1u << kp.block_warps) - 1);
-  const unsigned me = 1u << w.wid;
-  bool registered = false;
-  int old = 0;
-  if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
-  old = bcast(old);
-  if ((((unsigned)old) | me) == all) {
-    int got = 0;
-    if (w.lane == 0) got = atomicCAS(&bh->leader, -1, w.wid) == -1;
-    (void)bcast(got);
+  volatile WarpHdr* h = w.h;
+  const int me = 1 << w.wid;
+  if (w.lane == 0) {
+    __threadfence();
+    atomicSub(&kp.work->active, 1);
+    if (kp.local_steal) atomicOr(&bh->idle_mask, me);
   }
+  __syncwarp();
+  bool poller = false;
   for (int spin = 0;; ++spin) {
-    if ((spin & 1023) == 1023 && watchdog(kp, t0, "acquire")) return false;
-    int done = 0, leader = -1;
+    if ((spin & 63) == 63 && watchdog(kp, t0, "acquire")) return false;
+    int full = 0, done = 0;
     if (w.lane == 0) {
+      full = h->mail_full;
       done = *(volatile int*)&bh->done;
-      leader = *(volatile int*)&bh->leader;
     }
+    full = bcast(full);
     done = bcast(done);
-    leader = bcast(leader);
-    if (done) return false;
-    if (leader == w.wid) {
-      if (!kp.global_steal) {
-        if (w.lane == 0) atomicExch(&bh->done, 1);
-        __syncwarp();
-        return false;
-      }
-      StmBlockSlot* S = &kp.slots[blockIdx.x];
-      if (!registered) {
-        if (w.lane == 0) {
-          atomicAdd(&kp.work->idle_blocks, 1);
-          __threadfence();
-          atomicExch(&S->is_idle, 1);
-        }
-        __syncwarp();
-        registered = true;
-      }
-      int full = 0, nidle = 0;
+    if (full) {  // a donor of this block claimed this warp (cleared its bit, counted it active)
+      StmTask T;
       if (w.lane == 0) {
-        full = *(volatile int*)&S->mail_full;
-        nidle = *(volatile int*)&kp.work->idle_blocks;
+        __threadfence_block();
+        read_task(&h->mail, T);
+        h->mail_full = 0;
+        h->steal_fails = 0;
+        if (poller) {
+          if (kp.global_steal) atomicSub(&kp.work->deficit, 1);
+          atomicExch(&bh->poller, -1);
+        }
       }
-      full = bcast(full);
-      nidle = bcast(nidle);
-      if (full) {
-        StmTask T;
-        if (w.lane == 0) {
-          __threadfence();
-          volatile StmTask* M = &S->mail;
-          T.level = M->level;
-          T.b = M->b;
-          T.e = M->e;
-          for (int j = 0; j < STM_KMAX; ++j) {
-            T.prefix[j] = M->prefix[j];
-            T.tv[j] = M->tv[j];
+      bcast_task(T);
+      adopt_task(kp, T);
+      return true;
+    }
+    if (done) return false;
+    int got = 0;
+    StmTask T;
+    if (w.lane == 0) {
+      if (!poller && atomicCAS(&bh->poller, -1, w.wid) == -1) {
+        poller = true;
+        if (kp.global_steal) atomicAdd(&kp.work->deficit, 1);
+      }
+      if (poller) {
+        volatile StmWork* vw = kp.work;
+        if (vw->started == kp.total_warps && vw->active == 0) {
+          atomicExch(&bh->done, 1);  // every warp of the grid is idle: nothing can appear any more
+          done = 1;
+        } else if (kp.global_steal && vw->pool_head < vw->pool_tail) {
+          // leave local availability first (a donor may have claimed this warp already)
+          const int old = kp.local_steal ? atomicAnd(&bh->idle_mask, ~me) : me;
+          if (old & me) {
+            if (pool_pop(kp, T)) {  // (the queued task's unit of `active` is now this warp's)
+              got = 1;
+              h->steal_fails = 0;
+              atomicExch(&bh->poller, -1);  // (deficit: this poller leaves, one task less: net 0)
+            } else if (kp.local_steal) {
+              atomicOr(&bh->idle_mask, me);
+            }
           }
-          atomicExch(&S->mail_full, 0);
-          atomicExch(&S->is_idle, 0);
-          // leave the idle set before giving up leadership, so no other warp can
-          // see a full mask (and re-register the block) while this one works
-          atomicAnd(&bh->idle_mask, (int)~me);
-          __threadfence_block();
-          atomicExch(&bh->leader, -1);
         }
-        T.level = bcast(T.level);
-        T.b = bcast(T.b);
-        T.e = bcast(T.e);
-        for (int j = 0; j < STM_KMAX; ++j) {
-          T.prefix[j] = bcast(T.prefix[j]);
-          T.tv[j] = (int16_t)bcast(T.tv[j]);
-        }
-        adopt_task(kp, T);
-        return true;
-      }
-      if (nidle >= (int)gridDim.x) {
-        if (w.lane == 0) atomicExch(&bh->done, 1);
-        __syncwarp();
-        return false;
-      }
-    } else if (kp.local_steal) {
-      // leave the idle set while trying, so the block is never declared idle
-      // while a stolen task is in flight
-      if (w.lane == 0) atomicAnd(&bh->idle_mask, (int)~me);
-      __syncwarp();
-      if (try_local_steal(kp)) {
-        if (w.lane == 0) w.h->steal_fails = 0;
-        return true;
-      }
-      if (w.lane == 0) w.h->steal_fails = min(w.h->steal_fails + 1, kp.backoff_max);
-      if (w.lane == 0) old = atomicOr(&bh->idle_mask, (int)me);
-      old = bcast(old);
-      if ((((unsigned)old) | me) == all) {
-        if (w.lane == 0) atomicCAS(&bh->leader, -1, w.wid);
-        __syncwarp();
       }
     }
-    if (w.lane == 0) __nanosleep(32u << w.h->steal_fails);  // back off while nothing can be stolen
+    poller = __shfl_sync(FULLMASK, (int)poller, 0) != 0;
+    done = bcast(done);
+    got = bcast(got);
+    if (done) return false;
+    if (got) {
+      bcast_task(T);
+      adopt_task(kp, T);
+      return true;
+    }
+    if (w.lane == 0) {
+      __nanosleep(32u << h->steal_fails);  // back off while no work arrives
+      h->steal_fails = min(h->steal_fails + 1, kp.backoff_max);
+    }
     __syncwarp();
   }
 }
@@ -1749,13 +1823,13 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
   const int lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     bh->idle_mask = 0;
-    bh->leader = -1;
+    bh->poller = -1;
     bh->done = 0;
   }
   for (int i = threadIdx.x; i < 256; i += blockDim.x) bh->lab2slot[i] = kp.lab2slot[i];
   W w = make_w(kp);
   if (lane == 0) {
-    w.h->lock = 0;
+    w.h->mail_full = 0;
     w.h->L = 0;
     w.h->root_it = 0;
     w.h->root_end = 0;
@@ -1763,12 +1837,19 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     w.h->donate_tick = 0;
     w.h->steal_fails = 0;
     w.h->first_dry = 0;
+    w.h->gchk = 0;
+    w.h->deep = 0;
+    w.h->wd0 = gtimer();
     for (int i = 0; i < STM_KMAX; ++i) {
       w.h->nsib[i] = 0;
       w.h->cur[i] = 0;
       w.h->it[i] = 0;
       w.h->end[i] = 0;
     }
+    // termination accounting (acquire_work): this warp is active, then it has started
+    atomicAdd(&kp.work->active, 1);
+    __threadfence();
+    atomicAdd(&kp.work->started, 1);
   }
   __syncthreads();
 
@@ -1777,16 +1858,15 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
   const bool fused = !STM_MULTI && P.count_mode == STM_COUNT_FUSED;
   const long long t0 = clock64();
   const long long wd0 = gtimer();
-#if STM_PROFILE
-  long long prof_task0 = clock64();
-#endif
   unsigned iter = 0;
   for (;;) {
-    if ((++iter & 255) == 0 && watchdog(kp, wd0, "main")) break;
+    if ((++iter & 15) == 0 && watchdog(kp, wd0, "main")) break;
+    // local work sharing: a busy warp serves the idle warps of its block (one shared-
+    // memory load per iteration; the split runs only when a warp is waiting)
+    PROF_CHK()
+    if (kp.local_steal && waiting_warps(w)) share_local(kp);
     int L = w.h->L;
     if (L == 0) {
-      const bool lk = stealing(w);
-      if (lk) lock_ws(w, w.h);
       PROF_BEGIN(0)
       int m = gather_roots(w);
       PROF_END(0, m)
@@ -1807,7 +1887,6 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
         set_sibling(w, 1, 0);
         PROF_END(1, 1)
         if (k == 2) {
-          if (lk) unlock_ws(w, w.h);
           frame_count(w, m);  // counts N(root) per root
           continue;
         }
@@ -1815,23 +1894,19 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
         if (w.lane == 0) w.h->L = 1;
         __syncwarp();
       }
-      if (lk) unlock_ws(w, w.h);
       if (m == 0) {
         // instrumented launches: time spent acquiring work (cursor, stealing, idle
         // waiting) vs the warp's whole lifetime -> idle/stealing fraction (north_star)
         const long long ta = (STM_INSTR && kp.count_bytes) ? clock64() : 0;
 #if STM_PROFILE
-        // longest task (root chunk or stolen work) held by one warp: the critical path
-        if (lane == 0 && prof_task0) {
-          const unsigned long long d = (unsigned long long)(clock64() - prof_task0);
-          atomicMax(&kp.work->prof[3 * STM_PROF_N + 4 + STM_PROF_LVL - 2], d);
-        }
+        if (lane == 0) prof_timeline(w);  // busy until now
 #endif
         PROF_BEGIN(7)
         const bool got = acquire_work(kp, wd0);
         PROF_END(7, got)
 #if STM_PROFILE
-        prof_task0 = clock64();
+        w.prof_chk = 0;  // idle time is not a busy interval
+        w.prof_g = 0;
 #endif
         if (STM_INSTR && kp.count_bytes) w.idle_cyc += (unsigned long long)(clock64() - ta);
         if (!got) break;
@@ -1843,11 +1918,8 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     if (F == k - 2 && mvert(w, vert_of(w, F, w.h->cur[F])).n_build == 0 && w.h->cur[F] < w.h->nsib[F]) {
       fused_count_multi(w, F);
       if (w.h->cur[F] < w.h->nsib[F]) continue;  // stopped at a child that builds sets
-      const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
-      if (lk) lock_ws(w, w.h);
-      // (reads above are ordered before this write by a full-warp collective)
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
-      if (lk) unlock_ws(w, w.h);
       __syncwarp();
       continue;
     }
@@ -1858,23 +1930,18 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       fused_count(w, F);
 #endif
       PROF_END(5, 0)
-      const bool lk = locked_frame(w, F) || locked_frame(w, F - 1);
-      if (lk) lock_ws(w, w.h);
-      // (reads above are ordered before this write by a full-warp collective)
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
-      if (lk) unlock_ws(w, w.h);
       __syncwarp();
       continue;
     }
-    const bool lk = locked_frame(w, F);
-    // donors look for idle blocks at frames < detect_level (they donate only work of
+    // donors look at the pool's demand at frames < detect_level (they donate only work of
     // frames < stop_level: pick_split)
-    if (kp.global_steal && F < kp.detect_level) {
+    if (pool_wanted(w) && kp.global_steal && F < kp.detect_level) {
       PROF_BEGIN(6)
-      maybe_donate(kp);
+      maybe_push(kp);
       PROF_END(6, 0)
     }
-    if (lk) lock_ws(w, w.h);
     int m = 0;
     bool back = false;
     for (;;) {
@@ -1909,10 +1976,8 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
       if (w.lane == 0) w.h->L = F - 1;
       __syncwarp();
-      if (lk) unlock_ws(w, w.h);
       continue;
     }
-    if (lk) unlock_ws(w, w.h);
     // build frame F+1 from the batch
     PROF_BEGIN(3)
     m = build_nodes(w, F, m, true);
@@ -1924,9 +1989,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       PROF_END(4, m)
       continue;
     }
-    const bool lk2 = locked_frame(w, F + 1);
-    if (lk2) lock_ws(w, w.h);
-    // (reads above are ordered before this write by a full-warp collective)
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
     if (w.lane == 0) {
 #if STM_MULTI
       const int sv = vert_of(w, F, w.h->cur[F]);
@@ -1944,7 +2007,6 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     // (reads above are ordered before this write by a full-warp collective)
     if (w.lane == 0) w.h->L = F + 1;
     __syncwarp();
-    if (lk2) unlock_ws(w, w.h);
   }
   if (lane == 0 && w.cnt) atomicAdd(&kp.work->count, w.cnt);
 #if STM_PROFILE
@@ -1956,6 +2018,8 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
     }
     const long long now = clock64();
     atomicAdd(&kp.work->prof[3 * STM_PROF_N], (unsigned long long)(now - t0));
+    prof_timeline(w);
+    prof_timeline_flush(w);
     // tail shape (clock64 is per SM; SMs start within a few us of each other)
     atomicMax(&kp.work->prof[3 * STM_PROF_N + 1], (unsigned long long)(now - t0));
     const long long fd = w.h->first_dry;

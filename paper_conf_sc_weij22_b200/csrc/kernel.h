@@ -53,13 +53,24 @@ struct StmTask {
 #define STM_PROF_N 12
 // STM_PROFILE builds also keep, per level l (0..7) and kind (0 pre-test, 1 set build,
 // 2 count), the triple (warp cycles, combined operations, driven elements)
-#define STM_PROF_LVL (3 * 3 * 8 + 2)  // + (longest single task in cycles, its start time)
+#define STM_PROF_LVL (3 * 3 * 8 + 2)  // + (longest busy interval between sharing checks, spare)
+// STM_PROFILE builds also keep a timeline: busy warp-nanoseconds per 0.5 ms bucket of the
+// launch (%globaltimer since each warp's start), 64 buckets
+#define STM_PROF_TL 64
+#define STM_PROF_TL_NS 500000
+#define STM_PROF_SIZE (3 * STM_PROF_N + 4 + STM_PROF_LVL + STM_PROF_TL)
 
 // Device-resident scheduler state of one launch (zeroed before every launch).
 struct StmWork {
   unsigned long long count;       // result accumulator (mod 2^64)
-  int32_t idle_blocks;            // blocks registered idle (Fig. 6 is_idle count)
+  // Termination and the grid-wide task pool (kernel.cu acquire_work): `active` counts busy
+  // warps + queued pool tasks + claimed local donations; once every warp has started
+  // (`started` == all warps) and `active` is 0 no work can appear any more.  `deficit` =
+  // block pollers waiting for pool work - queued tasks: a donor pushes only after claiming
+  // a unit of it, so the pool never holds more tasks than there are blocks.
+  int32_t active, started, deficit;
   int32_t overflow;               // 1: a capacity check failed, 2: the watchdog expired (no count)
+  unsigned long long pool_head, pool_tail;  // tasks popped / pushed so far (tickets)
   unsigned long long n_local_steals, n_global_steals, n_chunks;
   unsigned long long n_peer_chunks;  // chunks taken from peer ranks' cursors
   unsigned int blocks_done;          // blocks that finished (the last one writes the async result)
@@ -70,16 +81,15 @@ struct StmWork {
   unsigned long long idle_cycles;  // sum over warps of cycles spent acquiring work (instrumented)
   unsigned long long warp_cycles;  // sum over warps of their lifetime in cycles (instrumented)
   unsigned long long list_n;       // listing build: embeddings found (slots taken) so far
-  unsigned long long prof[3 * STM_PROF_N + 4 + STM_PROF_LVL];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
+  unsigned long long prof[STM_PROF_SIZE];  // STM_PROFILE builds: (cycles, calls, items) per phase, summed
                                                 // lifetime, max lifetime, summed / max time cursors ran dry
 };
 
-struct StmBlockSlot {             // per block, global memory (Fig. 6)
-  int32_t is_idle;                // 0 busy, 1 idle & waiting, 2 claimed by a donor
-  int32_t mail_full;              // 1 when `mail` holds a task for this block
-  int32_t pad[2];
-  StmTask mail;
+struct StmPoolSlot {              // one slot of the grid-wide task pool (64 bytes)
+  int32_t seq;                    // 2r: free for the r-th round of tickets on this slot, 2r+1: holds it
+  StmTask task;
 };
+static_assert(sizeof(StmPoolSlot) == 64, "pool slot layout");
 
 struct StmKParams {
   StmPlan plan;
@@ -98,6 +108,10 @@ struct StmKParams {
   // handed out as several independent pieces from the start.  NULL: root space = vertex ids.
   const int2* entries;
   int32_t root_split;
+  // Work-balanced chunks (stm_tuning.chunk_cost): chunk c is root-space positions
+  // [chunk_bounds[c], chunk_bounds[c + 1]); NULL: fixed chunks of `chunk` positions.
+  const int32_t* chunk_bounds;
+  int64_t n_chunks;
   int64_t n;                      // root space end: roots are [root_lo, n)
   int64_t root_lo;
   int32_t* list_out;              // listing build: [list_cap][k] rows (pattern-vertex order)
@@ -106,7 +120,9 @@ struct StmKParams {
   int32_t block_warps;
   int32_t* arena;                 // [total_warps][n_nodes][cap]
   StmWork* work;
-  StmBlockSlot* slots;            // [gridDim.x]
+  StmPoolSlot* pool;              // [pool_mask + 1] task pool (global work sharing)
+  int32_t pool_mask, pool_shift;  // capacity - 1, log2(capacity)
+  int32_t total_warps;            // warps of the launch (termination: StmWork::started)
   unsigned long long* per_root;   // [n] or NULL (indexed by the caller's vertex id)
   const int32_t* root_map;        // counting id -> caller's id (degree-ranked copy), or NULL
   unsigned long long* cursors[8]; // chunk cursors (own rank + optional peers)

@@ -24,11 +24,12 @@
 #define STM_BITMAP_AUTO_MIN_DEGREE 64
 #define STM_BITMAP_AUTO_BUDGET_MB 2048
 #define STM_L2_PERSIST_AUTO_MB 0   // measured neutral at 24-48 MiB, worse at 96 MiB on C5: off
+#define STM_CHUNK_COST_AUTO 512    // work-balanced root chunks (stm_tuning.chunk_cost)
 #define STM_ROOT_SPLIT_AUTO 512    // root splitting piece size (stm_tuning.root_split; measured 32..512 on C2-C5)
 
 static thread_local char g_err[1024] = "";
 static thread_local stm_launch_info g_info = {};
-static thread_local uint64_t g_prof[3 * STM_PROF_N + 4 + STM_PROF_LVL] = {};
+static thread_local uint64_t g_prof[STM_PROF_SIZE] = {};
 
 stm_status stm_fail(stm_status s, const char* fmt, ...) {
   va_list ap;
@@ -50,7 +51,7 @@ namespace {
 struct Scratch {
   int* arena = nullptr;
   size_t arena_bytes = 0;
-  void* state = nullptr;  // StmWork + cursor + StmBlockSlot[grid]
+  void* state = nullptr;  // StmWork + cursor + StmPoolSlot[pool capacity]
   size_t state_bytes = 0;
 };
 
@@ -112,6 +113,12 @@ struct stm_graph {
     int64_t n = 0;
   };
   std::map<std::pair<int, int>, RootEntries> entries;
+  // work-balanced chunk bounds per (numbering, piece size or -1 = vertex ids, chunk cost)
+  struct ChunkBounds {
+    int32_t* d = nullptr;
+    int64_t n = 0;  // chunks (d has n + 1 entries)
+  };
+  std::map<std::tuple<int, int, int>, ChunkBounds> chunks;
   // degree / label statistics of the graph (NEXT-2 cost model), computed at load
   bool has_stats = false;
   stm_graph_stats stats;
@@ -336,6 +343,82 @@ static const stm_graph::RootEntries* ensure_entries(stm_graph* g, bool ranked, i
   }
   E.n = total;
   return &E;
+}
+
+// estimated cost of root-space position e: 1 + its level-1 candidate-list length (the
+// piece of its root's neighbour list when entries are used)
+__global__ void chunk_cost_fill(const int64_t* rp, const int2* ent, int64_t ne, int T, int64_t* cost) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x) {
+    const int v = ent ? ent[e].x : (int)e;
+    const int64_t d = rp[v + 1] - rp[v];
+    const int64_t len = ent ? min((int64_t)T, d - (int64_t)ent[e].y * T) : d;
+    cost[e] = 1 + max(len, (int64_t)0);
+  }
+}
+// position e starts a chunk iff its exclusive cost prefix lies in another multiple of C than e-1's
+__global__ void chunk_flag_fill(const int64_t* pre, int64_t ne, int64_t C, int32_t* flag) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x)
+    flag[e] = (e == 0 || pre[e] / C != pre[e - 1] / C) ? 1 : 0;
+}
+__global__ void chunk_scatter(const int32_t* flag, const int32_t* pos, int64_t ne, int32_t* out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x)
+    if (flag[e]) out[pos[e]] = (int32_t)e;
+}
+
+// Chunk bounds over the root space [0, ne) (entries E or vertex ids): consecutive positions
+// grouped until their cost reaches C.  Caller holds g->mu.  NULL on any failure (speed only:
+// the launch then uses fixed chunks).
+static const stm_graph::ChunkBounds* ensure_chunks(stm_graph* g, bool ranked, const stm_graph::RootEntries* E,
+                                                   int T, int C) {
+  const auto key = std::make_tuple(ranked ? 1 : 0, E ? T : -1, C);
+  auto it = g->chunks.find(key);
+  if (it != g->chunks.end()) return it->second.d ? &it->second : nullptr;
+  stm_graph::ChunkBounds& B = g->chunks[key];
+  const int64_t ne = E ? E->n : g->n;
+  if (ne < 1 || ne >= INT32_MAX || C < 1) return nullptr;
+  const int64_t* rp = ranked ? g->d_rrow_ptr : g->d_row_ptr;
+  int64_t* cost = nullptr;
+  int32_t *flag = nullptr, *pos = nullptr;
+  void* temp = nullptr;
+  size_t tb = 0, tb2 = 0;
+  const unsigned grid = (unsigned)std::min<int64_t>((ne + 255) / 256, 4096);
+  cudaError_t e = cudaMalloc(&cost, sizeof(int64_t) * ne);
+  if (e == cudaSuccess) e = cudaMalloc(&flag, sizeof(int32_t) * ne);
+  if (e == cudaSuccess) e = cudaMalloc(&pos, sizeof(int32_t) * ne);
+  if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(nullptr, tb, cost, cost, (int)ne);
+  if (e == cudaSuccess) e = cub::DeviceScan::ExclusiveSum(nullptr, tb2, flag, pos, (int)ne);
+  if (e == cudaSuccess) e = cudaMalloc(&temp, std::max<size_t>(std::max(tb, tb2), 16));
+  if (e == cudaSuccess) {
+    chunk_cost_fill<<<grid, 256>>>(rp, E ? E->d : nullptr, ne, T, cost);
+    e = cub::DeviceScan::ExclusiveSum(temp, tb, cost, cost, (int)ne);
+  }
+  if (e == cudaSuccess) {
+    chunk_flag_fill<<<grid, 256>>>(cost, ne, (int64_t)C, flag);
+    e = cub::DeviceScan::ExclusiveSum(temp, tb2, flag, pos, (int)ne);
+  }
+  int32_t last[2] = {0, 0};
+  if (e == cudaSuccess) e = cudaMemcpy(&last[0], pos + ne - 1, sizeof(int32_t), cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(&last[1], flag + ne - 1, sizeof(int32_t), cudaMemcpyDeviceToHost);
+  const int64_t nc = (int64_t)last[0] + last[1];
+  if (e == cudaSuccess) e = cudaMalloc(&B.d, sizeof(int32_t) * (nc + 1));
+  if (e == cudaSuccess) {
+    chunk_scatter<<<grid, 256>>>(flag, pos, ne, B.d);
+    const int32_t end = (int32_t)ne;
+    e = cudaMemcpy(B.d + nc, &end, sizeof end, cudaMemcpyHostToDevice);
+  }
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  cudaFree(cost);
+  cudaFree(flag);
+  cudaFree(pos);
+  cudaFree(temp);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    cudaFree(B.d);
+    B.d = nullptr;
+    return nullptr;
+  }
+  B.n = nc;
+  return &B;
 }
 
 static void free_hub(stm_graph::HubBitmaps& h) {
@@ -629,6 +712,7 @@ extern "C" stm_status stm_graph_free(stm_graph* g) {
   cudaFree(g->d_rout_start);
   for (auto& kv : g->hubs) free_hub(kv.second);
   for (auto& kv : g->entries) cudaFree(kv.second.d);
+  for (auto& kv : g->chunks) cudaFree(kv.second.d);
   delete g;
   return STM_OK;
 }
@@ -639,7 +723,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->local_steal = 1;
   t->global_steal = 1;
   t->stop_level = 2;
-  t->detect_level = 2;
+  t->detect_level = 8;  // donors look at the pool's demand at every frame (measured)
   t->unroll = 0;      // auto: 32 with the 40-register kernel, 16 with the 64-register one (measured)
   t->occupancy = 0;   // auto: 40-register kernel when the CSR does not fit in half the L2
   t->root_order = 0;  // auto
@@ -685,6 +769,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.backoff_max < 0 || t.backoff_max > 12) return stm_fail(STM_EINVAL, "backoff_max %d not in 0..12", t.backoff_max);
   if (t.carveout_pct < -1 || t.carveout_pct > 100) return stm_fail(STM_EINVAL, "carveout_pct %d", t.carveout_pct);
   if (t.root_split < -1) return stm_fail(STM_EINVAL, "root_split %d", t.root_split);
+  if (t.chunk_cost < -1) return stm_fail(STM_EINVAL, "chunk_cost %d", t.chunk_cost);
   if (d_result && ((uintptr_t)d_result & 7)) return stm_fail(STM_EINVAL, "d_result not 8-byte aligned");
   const StmPlan& P = p->dev;
   if (!p->labels.empty() && !g->d_labels) {
@@ -727,12 +812,25 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     g_info.hubs = hb->n_hubs;
     // root splitting (stm_tuning.root_split): not for listing pages, which are root-id ranges
     const int T = t.root_split == 0 ? STM_ROOT_SPLIT_AUTO : t.root_split;
+    const stm_graph::RootEntries* E = nullptr;
     if (!la && T > 0) {
-      const stm_graph::RootEntries* E = ensure_entries(g, use_rank, T);
+      E = ensure_entries(g, use_rank, T);
       if (E) {
         kp.entries = E->d;
         kp.root_split = T;
         kp.n = E->n;
+      }
+    }
+    // work-balanced chunks (stm_tuning.chunk_cost): not for listing pages (root-id ranges)
+    // auto: at most STM_CHUNK_COST_AUTO, and at least ~8 chunks per resident warp (48 per SM)
+    const int64_t c_auto = (g->n + g->nnz) / (8ll * 48 * std::max(1, g->num_sms));
+    const int C = t.chunk_cost == 0 ? (int)std::max<int64_t>(16, std::min<int64_t>(STM_CHUNK_COST_AUTO, c_auto))
+                                    : t.chunk_cost;
+    if (!la && C > 0) {
+      const stm_graph::ChunkBounds* B = ensure_chunks(g, use_rank, E, T, C);
+      if (B) {
+        kp.chunk_bounds = B->d;
+        kp.n_chunks = B->n;
       }
     }
   }
@@ -788,7 +886,8 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     }
   }
   glock.unlock();
-  kp.root_batch = std::max(1, std::min(STM_RMAX, root_chunk));
+  // roots gathered per frame-1 batch: with work-balanced chunks a light chunk holds many roots
+  kp.root_batch = (kp.chunk_bounds && t.root_chunk == 0) ? STM_RMAX : std::max(1, std::min(STM_RMAX, root_chunk));
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
     return stm_fail(STM_EINVAL, "hash_slots %d: 0 or a power of two in 64..4096", t.hash_slots);
@@ -813,7 +912,10 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   const int grid = bps * g->num_sms;
   const int64_t warps = (int64_t)grid * t.block_warps;
   const size_t arena_bytes = (size_t)warps * (size_t)P.n_nodes * (size_t)kp.cap * sizeof(int32_t);
-  const size_t state_bytes = sizeof(StmWork) + 64 + sizeof(StmBlockSlot) * (size_t)grid;
+  // task pool: never more tasks than blocks (StmWork::deficit), capacity 2 * grid rounded up
+  int pool_shift = 6;
+  while ((1 << pool_shift) < 2 * grid) ++pool_shift;
+  const size_t state_bytes = sizeof(StmWork) + 64 + sizeof(StmPoolSlot) * ((size_t)1 << pool_shift);
 
   Scratch* S;
   {
@@ -840,10 +942,12 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   StmWork* work = (StmWork*)S->state;
   unsigned long long* own_cursor = (unsigned long long*)((char*)S->state + sizeof(StmWork));
-  StmBlockSlot* slots = (StmBlockSlot*)((char*)S->state + sizeof(StmWork) + 64);
   kp.arena = S->arena;
   kp.work = work;
-  kp.slots = slots;
+  kp.pool = (StmPoolSlot*)((char*)S->state + sizeof(StmWork) + 64);
+  kp.pool_shift = pool_shift;
+  kp.pool_mask = (1 << pool_shift) - 1;
+  kp.total_warps = (int)warps;
   kp.per_root = d_per_root;
   if (shard) {
     kp.rank = shard->rank;
@@ -1011,7 +1115,7 @@ stm_status stm_launch_merged(const stm_graph* g, const stm_merged& m, const stm_
 
 extern "C" stm_status stm_last_profile(uint64_t* out, int n) {
   if (!out || n < 0) return stm_fail(STM_EINVAL, "NULL out");
-  for (int i = 0; i < n && i < 3 * STM_PROF_N + 4 + STM_PROF_LVL; ++i) out[i] = g_prof[i];
+  for (int i = 0; i < n && i < STM_PROF_SIZE; ++i) out[i] = g_prof[i];
   return STM_OK;
 }
 

@@ -43,7 +43,7 @@ class stm_tuning(ctypes.Structure):
                                                "instrument", "hash_slots", "vertex_order",
                                                "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
                                                "l2_persist_mb", "drive_ratio", "narrow_split", "watchdog_ms",
-                                               "backoff_max", "carveout_pct", "root_split")]
+                                               "backoff_max", "carveout_pct", "root_split", "chunk_cost")]
 
 
 class stm_shard(ctypes.Structure):
@@ -383,8 +383,9 @@ PROF_PHASES = ["gather_roots", "root_sibling", "gather_batch", "build_nodes", "f
 def stm_last_profile() -> dict:
     N = 3 * len(PROF_PHASES) + 4
     NL = 3 * 3 * 8 + 2
-    out = (ctypes.c_uint64 * (N + NL))()
-    _check(lib.stm_last_profile(out, N + NL))
+    NT = 64  # timeline buckets (kernel.h STM_PROF_TL, 0.5 ms each)
+    out = (ctypes.c_uint64 * (N + NL + NT))()
+    _check(lib.stm_last_profile(out, N + NL + NT))
     d = {ph: {"cycles": out[3 * i], "calls": out[3 * i + 1], "items": out[3 * i + 2]}
          for i, ph in enumerate(PROF_PHASES)}
     d["lifetime_cycles"] = out[N - 4]
@@ -397,6 +398,7 @@ def stm_last_profile() -> dict:
                 lv[f"{kn}@L{lvl}"] = {"cycles": c, "ops": j, "elements": e}
     d["levels"] = lv
     d["max_task_cycles"] = out[N + NL - 2]
+    d["timeline_busy_warps"] = [out[N + NL + i] / 5e5 for i in range(NT)]  # mean busy warps per 0.5 ms
     return d
 
 

@@ -131,6 +131,12 @@ TUNINGS = [
     dict(root_split=-1), dict(root_split=1), dict(root_split=3, root_chunk=5, stop_level=3),
     dict(root_split=2, vertex_order=1, root_order=2), dict(root_split=4, root_chunk=1, unroll=2),
     dict(backoff_max=1, carveout_pct=-1), dict(backoff_max=12, carveout_pct=50),
+    # donation at every frame (split kinds 2 and 3 below frame 1), small batches, one big block
+    dict(stop_level=8, root_chunk=1, unroll=2), dict(stop_level=8, detect_level=8, unroll=1, root_split=1),
+    dict(stop_level=8, block_warps=32, blocks_per_sm=1, root_chunk=1),
+    # work-balanced chunks: off, one position per chunk, descending, one huge chunk
+    dict(chunk_cost=-1), dict(chunk_cost=1), dict(chunk_cost=64, root_order=2, root_chunk=3),
+    dict(chunk_cost=1 << 30, root_split=-1), dict(chunk_cost=40, vertex_order=1, root_split=-1),
 ]
 
 

@@ -28,7 +28,8 @@ out = {
     "kernel_ms": val("gpu__time_duration.sum"),
     "warp_execution_efficiency": val("smsp__thread_inst_executed_per_inst_executed.ratio") / 32.0,
     "dram_read_gbs": val("dram__bytes_read.sum.per_second") * rate[d["dram__bytes_read.sum.per_second"]["unit"]],
-    "l2_gbs": val("lts__t_bytes.sum.per_second") * rate[d["lts__t_bytes.sum.per_second"]["unit"]],
+    "l2_gbs": (val("lts__t_bytes.sum.per_second") * rate[d["lts__t_bytes.sum.per_second"]["unit"]]
+               if "lts__t_bytes.sum.per_second" in d else val("lts__t_sectors.sum.per_second") * 32.0),  # sector/ns * 32 B
     "l2_hit_pct": val("lts__t_sector_hit_rate.pct"), "l1_hit_pct": val("l1tex__t_sector_hit_rate.pct"),
     "warps_active_pct": val("sm__warps_active.avg.pct_of_peak_sustained_active"),
     "top_stalls_per_issue": d["stalls_per_issue"],

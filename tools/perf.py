@@ -39,7 +39,10 @@ for spec in specs:
             tail = prof.pop("tail")
             lv = prof.pop("levels")
             mt = prof.pop("max_task_cycles")
-            print(f"   longest single task (critical path): {mt / 1.9e6:.2f} ms", flush=True)
+            tl = prof.pop("timeline_busy_warps")
+            last = max([i for i, x in enumerate(tl) if x > 0] or [0])
+            print("   busy warps per 0.5 ms: " + " ".join(f"{x:.0f}" for x in tl[:last + 1]), flush=True)
+            print(f"   longest busy interval between work-sharing checks (indivisible unit): {mt / 1.9e6:.2f} ms", flush=True)
             nw = info["grid"] * info["block_threads"] // 32
             print(f"   tail: mean lifetime {L / nw / 1.9e6:.2f} ms, max {tail['max_lifetime'] / 1.9e6:.2f} ms, "
                   f"cursors dry at mean {tail['sum_dry'] / nw / 1.9e6:.2f} ms / max {tail['max_dry'] / 1.9e6:.2f} ms "
