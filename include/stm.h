@@ -140,6 +140,12 @@ stm_status stm_plan_describe(const stm_plan* p, char* buf, size_t len);
 /* stm_plan_info -- pattern size, number of materialised set nodes, |Aut_L(Q)|. Any out may be NULL. */
 stm_status stm_plan_info(const stm_plan* p, int* k, int* n_sets, int64_t* aut_size);
 
+/* stm_plan_raw -- the compiled device plan (the StmPlan record the kernel interprets,
+ * paper_conf_sc_weij22_b200/csrc/plan.h) as bytes: *size receives its size; buf (len bytes,
+ * may be NULL to query the size) receives a copy.  Used to build plan-specialised kernels
+ * (tools/cplan.py) and by tests.  STM_EINVAL if buf is too small. */
+stm_status stm_plan_raw(const stm_plan* p, void* buf, size_t len, size_t* size);
+
 stm_status stm_plan_free(stm_plan* p);
 
 /* Tuning knobs: every setting changes speed only, never the count. NULL = defaults. */
@@ -211,6 +217,13 @@ typedef struct stm_tuning {
                              (min(512, (n + nnz) / (8 * 48 * SMs)), at least 16: ~8 chunks per warp),
                              -1 = off (fixed root_chunk roots per chunk).  Counting launches only (not
                              listing pages).  Speed only. */
+  int32_t jit;            /* plan-specialised kernels: the counting
+                             kernel is compiled once more for the plan (NVRTC, a few seconds at the first
+                             launch of each plan, cached for the process) with the plan and the frame as
+                             compile-time constants.  0 = auto (on; the generic kernel if the compile
+                             fails), 1 = required (STM_EUNSUPPORTED if it cannot be built), -1 = off.
+                             Counting launches only (not instrumented, listing or census launches).
+                             Speed only. */
 } stm_tuning;
 
 /* Fill t with the defaults. */
@@ -344,7 +357,7 @@ typedef struct stm_launch_info {
   int64_t merge_bytes;     /* merge-equivalent bytes W_merge; instrumented calls only */
   int64_t jobs;            /* set operations executed; instrumented calls only */
   int32_t ranked;          /* 1 = counted on the degree-ranked copy (stm_tuning.vertex_order) */
-  int32_t reserved;
+  int32_t jit;             /* 1 = the plan-specialised kernel ran (stm_tuning.jit), 0 = the generic one */
   int64_t idle_cycles;     /* sum over warps of SM cycles spent acquiring work (root cursor, stealing,
                               waiting idle); instrumented calls only */
   int64_t warp_cycles;     /* sum over warps of their lifetime in SM cycles; instrumented calls only.

@@ -503,6 +503,16 @@ extern "C" stm_status stm_plan_describe(const stm_plan* p, char* buf, size_t len
   return STM_OK;
 }
 
+extern "C" stm_status stm_plan_raw(const stm_plan* p, void* buf, size_t len, size_t* size) {
+  if (!p) return stm_fail(STM_EINVAL, "NULL plan");
+  if (size) *size = sizeof(StmPlan);
+  if (buf) {
+    if (len < sizeof(StmPlan)) return stm_fail(STM_EINVAL, "buffer of %zu bytes < %zu", len, sizeof(StmPlan));
+    memcpy(buf, &p->dev, sizeof(StmPlan));
+  }
+  return STM_OK;
+}
+
 extern "C" stm_status stm_plan_info(const stm_plan* p, int* k, int* n_sets, int64_t* aut) {
   if (!p) return stm_fail(STM_EINVAL, "NULL plan");
   if (k) *k = p->k;

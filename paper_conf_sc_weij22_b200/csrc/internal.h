@@ -38,3 +38,8 @@ struct stm_merged {
 // one persistent launch of the merged plan; counts[i] += count of pattern i
 stm_status stm_launch_merged(const stm_graph* g, const stm_merged& m, const stm_tuning* t, void* stream,
                              uint64_t* counts);
+
+// plan-specialised counting kernel of P for a register variant (jit.cpp): compiled with
+// NVRTC on first use and cached; NULL (with *err) if it cannot be built
+const void* stm_jit_kernel(const StmPlan& P, int variant, std::string* err);
+int stm_jit_cache_size();

@@ -24,6 +24,10 @@
 // PAPER.md:84) and inter-block stealing through per-block global mailboxes pushed
 // by busy donors (Sec. V-B, Fig. 6).  Stolen work is a task
 // (prefix, position range); the thief rebuilds the prefix's sets itself.
+#ifdef STM_NVRTC
+// plan-specialised JIT compile (runtime.cu jit_kernel, NVRTC): device code only
+#include "stm_nvrtc_prelude.h"
+#else
 #include <algorithm>
 #include <climits>
 #include <cmath>
@@ -32,6 +36,7 @@
 #include <cstdint>
 
 #include <cuda_runtime.h>
+#endif
 
 #include "kernel.h"
 
@@ -93,6 +98,9 @@
 #else
 #define STM_SYM(x) x
 #endif
+#ifndef STM_CPLAN
+#define STM_CPLAN 0         // 1: plan-specialised build: the plan is the compile-time record of
+#endif                      //    STM_CPLAN_HEADER (tools/cplan.py) instead of kp.plan
 #ifndef STM_DEBUG
 #define STM_DEBUG 0         // 1: watchdog state dumps (printf)
 #endif
@@ -212,8 +220,21 @@ struct W {
 
 extern __shared__ __align__(16) unsigned char stm_smem[];
 
+#if STM_CPLAN
+// The plan as a constant initialised global: every load from it at a constant offset folds
+// to an immediate (frame_step<F> makes the frame a constant, the node loops unroll).
+union StmPlanBytes {
+  unsigned char b[sizeof(StmPlan)];
+  StmPlan p;
+};
+#include STM_CPLAN_HEADER  // __device__ const StmPlanBytes kCPlan = {{...}};
+#define STM_PLAN_OF(kp) (kCPlan.p)
+#else
+#define STM_PLAN_OF(kp) ((kp).plan)
+#endif
+
 __device__ __forceinline__ W make_w(const StmKParams& kp) {
-  const StmPlan& P = kp.plan;
+  const StmPlan& P = STM_PLAN_OF(kp);
   W w;
   w.kp = &kp;
   w.P = &P;
@@ -1814,11 +1835,113 @@ __device__ __noinline__ bool acquire_work(const StmKParams& kp, long long t0) {
 
 }  // namespace
 
+// One main-loop iteration at frame F >= 1: the fused count of frame k-2, or the next
+// batch of frame F (gather -> build frame F+1 -> descend), or the backtrack.  FC >= 0:
+// F == FC is a compile-time constant (plan-specialised builds, STM_CPLAN: every plan
+// lookup indexed by the frame folds to a constant and the node loops unroll).
+template <int FC>
+__device__ __forceinline__ void frame_step(W& w, const StmKParams& kp, int Fr, int k, int U, bool fused) {
+  const int F = FC >= 0 ? FC : Fr;
+#if STM_MULTI
+  if (F == k - 2 && mvert(w, vert_of(w, F, w.h->cur[F])).n_build == 0 && w.h->cur[F] < w.h->nsib[F]) {
+    fused_count_multi(w, F);
+    if (w.h->cur[F] < w.h->nsib[F]) return;  // stopped at a child that builds sets
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+    if (w.lane == 0) w.h->L = F - 1;
+    __syncwarp();
+    return;
+  }
+#endif
+  if (fused && F == k - 2) {
+    PROF_BEGIN(5)
+#if !STM_MULTI
+    fused_count(w, F);
+#endif
+    PROF_END(5, 0)
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+    if (w.lane == 0) w.h->L = F - 1;
+    __syncwarp();
+    return;
+  }
+  // donors look at the pool's demand at frames < detect_level (they donate only work of
+  // frames < stop_level: pick_split)
+  if (pool_wanted(w) && kp.global_steal && F < kp.detect_level) {
+    PROF_BEGIN(6)
+    maybe_push(kp);
+    PROF_END(6, 0)
+  }
+  int m = 0;
+  bool back = false;
+  for (;;) {
+    if (w.h->cur[F] >= w.h->nsib[F]) { back = true; break; }
+    if (w.h->it[F] < w.h->end[F]) {
+      int Ub = U;
+#if STM_MULTI
+      {  // a frame that builds no set node has no per-sibling slice table: batch up to 32
+        int nb, ne, nst;
+        bset(w, F, w.h->cur[F], nb, ne, nst);
+        if (nb == ne) Ub = STM_RMAX;
+      }
+#endif
+      PROF_BEGIN(2)
+      m = gather_batch(w, F, Ub);
+      PROF_END(2, m)
+      if (m > 0) break;
+    }
+    int nu = w.h->cur[F] + 1;
+    if (nu >= w.h->nsib[F]) {
+      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+      if (w.lane == 0) w.h->cur[F] = nu;
+      __syncwarp();
+      back = true;
+      break;
+    }
+    PROF_BEGIN(8)
+    set_sibling(w, F, nu);
+    PROF_END(8, 1)
+  }
+  if (back) {
+    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+    if (w.lane == 0) w.h->L = F - 1;
+    __syncwarp();
+    return;
+  }
+  // build frame F+1 from the batch
+  PROF_BEGIN(3)
+  m = build_nodes(w, F, m, true);
+  PROF_END(3, m)
+  if (m == 0) return;  // every sibling of the batch was pruned: gather the next one
+  if (F + 1 == k - 1) {  // frame-count mode
+    PROF_BEGIN(4)
+    frame_count(w, m);
+    PROF_END(4, m)
+    return;
+  }
+  HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
+  if (w.lane == 0) {
+#if STM_MULTI
+    const int sv = vert_of(w, F, w.h->cur[F]);
+    w.h->pv[F + 1] = sv;
+    w.h->nr[F + 1] = m;
+    w.h->nsib[F + 1] = m * kp.mv[sv].n_children;
+#else
+    w.h->nsib[F + 1] = m;
+#endif
+  }
+  __syncwarp();
+  PROF_BEGIN(9)
+  set_sibling(w, F + 1, 0);
+  PROF_END(9, 1)
+  // (reads above are ordered before this write by a full-warp collective)
+  if (w.lane == 0) w.h->L = F + 1;
+  __syncwarp();
+}
+
 // ----------------------------------------------------------------------------
 // the kernel
 // ----------------------------------------------------------------------------
 __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
-  const StmPlan& P = kp.plan;
+  const StmPlan& P = STM_PLAN_OF(kp);
   BlockHdr* bh = (BlockHdr*)stm_smem;
   const int lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -1913,100 +2036,29 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
       }
       continue;
     }
-    const int F = L;
-#if STM_MULTI
-    if (F == k - 2 && mvert(w, vert_of(w, F, w.h->cur[F])).n_build == 0 && w.h->cur[F] < w.h->nsib[F]) {
-      fused_count_multi(w, F);
-      if (w.h->cur[F] < w.h->nsib[F]) continue;  // stopped at a child that builds sets
-      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-      if (w.lane == 0) w.h->L = F - 1;
-      __syncwarp();
-      continue;
-    }
+#if STM_CPLAN
+    switch (L) {  // a specialised copy per frame 1..k-2 (frames >= k-1 are never entered)
+      case 1: frame_step<1>(w, kp, L, k, U, fused); break;
+#if STM_CPLAN_K > 3
+      case 2: frame_step<2>(w, kp, L, k, U, fused); break;
 #endif
-    if (fused && F == k - 2) {
-      PROF_BEGIN(5)
-#if !STM_MULTI
-      fused_count(w, F);
+#if STM_CPLAN_K > 4
+      case 3: frame_step<3>(w, kp, L, k, U, fused); break;
 #endif
-      PROF_END(5, 0)
-      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-      if (w.lane == 0) w.h->L = F - 1;
-      __syncwarp();
-      continue;
-    }
-    // donors look at the pool's demand at frames < detect_level (they donate only work of
-    // frames < stop_level: pick_split)
-    if (pool_wanted(w) && kp.global_steal && F < kp.detect_level) {
-      PROF_BEGIN(6)
-      maybe_push(kp);
-      PROF_END(6, 0)
-    }
-    int m = 0;
-    bool back = false;
-    for (;;) {
-      if (w.h->cur[F] >= w.h->nsib[F]) { back = true; break; }
-      if (w.h->it[F] < w.h->end[F]) {
-        int Ub = U;
-#if STM_MULTI
-        {  // a frame that builds no set node has no per-sibling slice table: batch up to 32
-          int nb, ne, nst;
-          bset(w, F, w.h->cur[F], nb, ne, nst);
-          if (nb == ne) Ub = STM_RMAX;
-        }
+#if STM_CPLAN_K > 5
+      case 4: frame_step<4>(w, kp, L, k, U, fused); break;
 #endif
-        PROF_BEGIN(2)
-        m = gather_batch(w, F, Ub);
-        PROF_END(2, m)
-        if (m > 0) break;
-      }
-      int nu = w.h->cur[F] + 1;
-      if (nu >= w.h->nsib[F]) {
-        HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-        if (w.lane == 0) w.h->cur[F] = nu;
-        __syncwarp();
-        back = true;
-        break;
-      }
-      PROF_BEGIN(8)
-      set_sibling(w, F, nu);
-      PROF_END(8, 1)
+#if STM_CPLAN_K > 6
+      case 5: frame_step<5>(w, kp, L, k, U, fused); break;
+#endif
+#if STM_CPLAN_K > 7
+      case 6: frame_step<6>(w, kp, L, k, U, fused); break;
+#endif
+      default: break;
     }
-    if (back) {
-      HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-      if (w.lane == 0) w.h->L = F - 1;
-      __syncwarp();
-      continue;
-    }
-    // build frame F+1 from the batch
-    PROF_BEGIN(3)
-    m = build_nodes(w, F, m, true);
-    PROF_END(3, m)
-    if (m == 0) continue;  // every sibling of the batch was pruned: gather the next one
-    if (F + 1 == k - 1) {  // frame-count mode
-      PROF_BEGIN(4)
-      frame_count(w, m);
-      PROF_END(4, m)
-      continue;
-    }
-    HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
-    if (w.lane == 0) {
-#if STM_MULTI
-      const int sv = vert_of(w, F, w.h->cur[F]);
-      w.h->pv[F + 1] = sv;
-      w.h->nr[F + 1] = m;
-      w.h->nsib[F + 1] = m * kp.mv[sv].n_children;
 #else
-      w.h->nsib[F + 1] = m;
+    frame_step<-1>(w, kp, L, k, U, fused);
 #endif
-    }
-    __syncwarp();
-    PROF_BEGIN(9)
-    set_sibling(w, F + 1, 0);
-    PROF_END(9, 1)
-    // (reads above are ordered before this write by a full-warp collective)
-    if (w.lane == 0) w.h->L = F + 1;
-    __syncwarp();
   }
   if (lane == 0 && w.cnt) atomicAdd(&kp.work->count, w.cnt);
 #if STM_PROFILE
@@ -2057,12 +2109,23 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
 // Two register budgets of the same kernel (stm_tuning.occupancy): 64 registers ->
 // 32 resident warps per SM, or 40 registers (with spills) -> 48 warps per SM, which
 // hides more DRAM latency when the graph does not fit in L2 (measured).
-__global__ void __launch_bounds__(STM_MAXT, 1) STM_SYM(stm_count_kernel)(const __grid_constant__ StmKParams kp) {
+#ifdef STM_NVRTC
+#define STM_KLINK extern "C"  // JIT builds: unmangled names for cudaLibraryGetKernel
+#else
+#define STM_KLINK
+#endif
+#if !defined(STM_JIT_VARIANT) || STM_JIT_VARIANT == 1
+STM_KLINK __global__ void __launch_bounds__(STM_MAXT, 1) STM_SYM(stm_count_kernel)(const __grid_constant__ StmKParams kp) {
   stm_count_body(kp);
 }
-__global__ void __launch_bounds__(STM_OCC_MAXT, 1) STM_SYM(stm_count_kernel_occ)(const __grid_constant__ StmKParams kp) {
+#endif
+#if !defined(STM_JIT_VARIANT) || STM_JIT_VARIANT == 2
+STM_KLINK __global__ void __launch_bounds__(STM_OCC_MAXT, 1) STM_SYM(stm_count_kernel_occ)(const __grid_constant__ StmKParams kp) {
   stm_count_body(kp);
 }
+#endif
+
+#ifndef STM_NVRTC  // host side of the launch (never part of a JIT compile)
 
 static const void* STM_SYM(kernel_fn)(int variant) {
   return variant == 2 ? (const void*)STM_SYM(stm_count_kernel_occ) : (const void*)STM_SYM(stm_count_kernel);
@@ -2086,9 +2149,18 @@ int stm_smem_bytes_multi(int block_warps, int k, int n_regions) {
 }
 #endif
 
+int STM_SYM(stm_occupancy_fn)(const void* fn, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                              int* blocks_per_sm);
+int STM_SYM(stm_launch_fn)(const void* fn, const StmKParams& kp, int grid, void* stream);
+
 int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
                            int* blocks_per_sm) {
-  const void* fn = STM_SYM(kernel_fn)(variant);
+  return STM_SYM(stm_occupancy_fn)(STM_SYM(kernel_fn)(variant), block_warps, k, n_nodes, ht_slots, carveout,
+                                   blocks_per_sm);
+}
+
+int STM_SYM(stm_occupancy_fn)(const void* fn, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                              int* blocks_per_sm) {
   int smem = local_smem_bytes(block_warps, k, n_nodes, ht_slots);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
@@ -2116,7 +2188,10 @@ int STM_SYM(stm_occupancy)(int variant, int block_warps, int k, int n_nodes, int
 }
 
 int STM_SYM(stm_launch)(int variant, const StmKParams& kp, int grid, void* stream) {
-  const void* fn = STM_SYM(kernel_fn)(variant);
+  return STM_SYM(stm_launch_fn)(STM_SYM(kernel_fn)(variant), kp, grid, stream);
+}
+
+int STM_SYM(stm_launch_fn)(const void* fn, const StmKParams& kp, int grid, void* stream) {
   int smem = local_smem_bytes(kp.block_warps, kp.plan.k, kp.plan.n_nodes, kp.ht_slots);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return (int)e;
@@ -2146,3 +2221,4 @@ int STM_SYM(stm_launch)(int variant, const StmKParams& kp, int grid, void* strea
   e = cudaLaunchKernelExC(&cfg, fn, args);
   return (int)e;
 }
+#endif  // !STM_NVRTC

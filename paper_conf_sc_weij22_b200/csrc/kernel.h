@@ -1,9 +1,11 @@
 // kernel.h -- launch interface between the runtime (runtime.cu) and the persistent
 // matching kernel (kernel.cu).  Product code only.
 #pragma once
+#ifndef STM_NVRTC  // (JIT compiles get the fixed-width types from stm_nvrtc_prelude.h)
 #include <stdint.h>
 
 #include <cuda_runtime.h>  // int4
+#endif
 
 #include "plan.h"
 
@@ -145,6 +147,7 @@ struct StmKParams {
   unsigned long long* mcount;     // [n_patterns] counts (zeroed by the host)
 };
 
+#ifndef STM_NVRTC  // host-side launch interface (not part of a JIT compile)
 // 1 if the shared-memory hash-set path is compiled in (-DSTM_WITH_HASH=1)
 int stm_hash_compiled();
 // 1 if the drive_ratio operand choice is compiled in (-DSTM_DRIVE_RATIO=1)
@@ -160,6 +163,10 @@ int stm_launch_multi(int variant, const StmKParams& kp, int grid, void* stream);
 // max co-resident blocks per SM for the given block size
 // carveout: stm_tuning.carveout_pct (0 = auto, -1 = driver default, else percent)
 int stm_occupancy(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout, int* blocks_per_sm);
+// the same for a given kernel: a plan-specialised JIT kernel (cudaKernel_t), runtime.cu jit_kernel
+int stm_occupancy_fn(const void* fn, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
+                     int* blocks_per_sm);
+int stm_launch_fn(const void* fn, const StmKParams& kp, int grid, void* stream);
 int stm_occupancy_instr(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
                         int* blocks_per_sm);
 int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
@@ -167,3 +174,4 @@ int stm_occupancy_list(int variant, int block_warps, int k, int n_nodes, int ht_
 int stm_occupancy_multi(int variant, int block_warps, int k, int n_nodes, int ht_slots, int carveout,
                         int* blocks_per_sm);
 int stm_smem_bytes_multi(int block_warps, int k, int n_regions);
+#endif  // !STM_NVRTC

@@ -15,7 +15,9 @@
 // replaces the paper's (first-operand flag, op, dependency) triples
 // (self-contradictory in the extracted text; reading R7).
 #pragma once
+#ifndef STM_NVRTC
 #include <stdint.h>
+#endif
 
 #define STM_KMAX 8
 #define STM_MAX_NODES 32

@@ -770,6 +770,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.carveout_pct < -1 || t.carveout_pct > 100) return stm_fail(STM_EINVAL, "carveout_pct %d", t.carveout_pct);
   if (t.root_split < -1) return stm_fail(STM_EINVAL, "root_split %d", t.root_split);
   if (t.chunk_cost < -1) return stm_fail(STM_EINVAL, "chunk_cost %d", t.chunk_cost);
+  if (t.jit < -1 || t.jit > 1) return stm_fail(STM_EINVAL, "jit %d not in -1..1", t.jit);
   if (d_result && ((uintptr_t)d_result & 7)) return stm_fail(STM_EINVAL, "d_result not 8-byte aligned");
   const StmPlan& P = p->dev;
   if (!p->labels.empty() && !g->d_labels) {
@@ -904,8 +905,16 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
 
   int bps = 0;
   if (ma && (la || t.instrument)) return stm_fail(STM_EINVAL, "merged launches do not list or instrument");
-  int oe = (ma ? stm_occupancy_multi : la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(
-      variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps);
+  // plan-specialised kernel (jit.cpp; stm_tuning.jit) for plain counting launches
+  const void* jfn = nullptr;
+  if (!ma && !la && !t.instrument && t.jit >= 0) {
+    std::string jerr;
+    jfn = stm_jit_kernel(P, variant, &jerr);
+    if (!jfn && t.jit == 1) return stm_fail(STM_EUNSUPPORTED, "plan-specialised kernel: %s", jerr.c_str());
+  }
+  int oe = jfn ? stm_occupancy_fn(jfn, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps)
+               : (ma ? stm_occupancy_multi : la ? stm_occupancy_list : t.instrument ? stm_occupancy_instr : stm_occupancy)(
+                     variant, t.block_warps, P.k, P.n_nodes, t.hash_slots, t.carveout_pct, &bps);
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy (variant %d, %s build, %d warps): %s", variant, la ? "list" : t.instrument ? "instr" : "count", t.block_warps, cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
@@ -962,8 +971,9 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   }
   cudaStream_t st = (cudaStream_t)stream;
   CU(cudaMemsetAsync(S->state, 0, state_bytes, st));
-  int le = (ma ? stm_launch_multi : la ? stm_launch_list : t.instrument ? stm_launch_instr : stm_launch)(
-      variant, kp, grid, stream);
+  int le = jfn ? stm_launch_fn(jfn, kp, grid, stream)
+               : (ma ? stm_launch_multi : la ? stm_launch_list : t.instrument ? stm_launch_instr : stm_launch)(
+                     variant, kp, grid, stream);
   if (le != 0) return stm_fail(STM_ECUDA, "launch: %s", cudaGetErrorString((cudaError_t)le));
   g_info.grid = grid;
   g_info.block_threads = t.block_warps * 32;
@@ -972,6 +982,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   g_info.arena_bytes = (int64_t)arena_bytes;
   g_info.cap = kp.cap;
   g_info.ranked = use_rank ? 1 : 0;
+  g_info.jit = jfn ? 1 : 0;
   g_info.variant = variant;
   g_info.unroll = kp.unroll;
   if (h_count) {

@@ -28,7 +28,8 @@ EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_gra
            "stm_match_count_async", "stm_match_count_per_root", "stm_last_launch", "stm_last_profile", "stm_last_error",
            "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize", "stm_motif_catalog",
            "stm_motif_census", "stm_cursors_alloc", "stm_cursors_open", "stm_cursors_close", "stm_cursors_free",
-           "stm_cursors_reset", "stm_graph_get_stats", "stm_motif_census_launches", "stm_motif_merge_stats"]
+           "stm_cursors_reset", "stm_graph_get_stats", "stm_motif_census_launches", "stm_motif_merge_stats",
+           "stm_plan_raw"]
 
 
 class StmError(RuntimeError):
@@ -43,7 +44,7 @@ class stm_tuning(ctypes.Structure):
                                                "instrument", "hash_slots", "vertex_order",
                                                "bitmap_min_degree", "bitmap_budget_mb", "occupancy", "root_order",
                                                "l2_persist_mb", "drive_ratio", "narrow_split", "watchdog_ms",
-                                               "backoff_max", "carveout_pct", "root_split", "chunk_cost")]
+                                               "backoff_max", "carveout_pct", "root_split", "chunk_cost", "jit")]
 
 
 class stm_shard(ctypes.Structure):
@@ -56,7 +57,7 @@ class stm_launch_info(ctypes.Structure):
                 ("cap", ctypes.c_int32), ("arena_bytes", ctypes.c_int64), ("local_steals", ctypes.c_int64),
                 ("global_steals", ctypes.c_int64), ("chunks", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("merge_bytes", ctypes.c_int64), ("jobs", ctypes.c_int64), ("ranked", ctypes.c_int32),
-                ("reserved", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64),
+                ("jit", ctypes.c_int32), ("idle_cycles", ctypes.c_int64), ("warp_cycles", ctypes.c_int64),
                 ("hubs", ctypes.c_int64), ("variant", ctypes.c_int32), ("unroll", ctypes.c_int32),
                 ("peer_chunks", ctypes.c_int64)]
 
@@ -96,6 +97,7 @@ def _load():
         "stm_plan_describe": [vp, ctypes.c_char_p, sz],
         "stm_plan_info": [vp, ctypes.POINTER(i32), ctypes.POINTER(i32), P64],
         "stm_plan_free": [vp],
+        "stm_plan_raw": [vp, vp, sz, ctypes.POINTER(sz)],
         "stm_plan_first_vertex": [vp, ctypes.POINTER(i32)],
         "stm_match_count": [vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
         "stm_match_count_ex": [vp, vp, vp, vp, vp, ctypes.POINTER(ctypes.c_uint64)],
@@ -274,6 +276,15 @@ def stm_plan_first_vertex(p: int) -> int:
     u = ctypes.c_int()
     _check(lib.stm_plan_first_vertex(p, ctypes.byref(u)))
     return u.value
+
+
+def stm_plan_raw(p: int) -> bytes:
+    """The compiled device plan record (plan.h StmPlan) as bytes."""
+    n = ctypes.c_size_t()
+    _check(lib.stm_plan_raw(p, None, 0, ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value)
+    _check(lib.stm_plan_raw(p, buf, n.value, ctypes.byref(n)))
+    return buf.raw
 
 
 def stm_plan_free(p: int) -> None:

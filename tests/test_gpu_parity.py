@@ -199,8 +199,10 @@ def test_golden_config_counts():
         plan = stm.Plan(d["k"], d["edges"], d["labels"], restrictions=d["restrictions"], auto_restrict=False,
                         vertex_induced=d["vertex_induced"])
         assert stm.count(G, plan) == d["count"], cid
+        # the product default: the plan-specialised kernel (jit.cpp) of the compiler's own plan
         plan2 = stm.Plan(d["k"], d["edges"], d["labels"], vertex_induced=d["vertex_induced"])
-        assert stm.count(G, plan2) == d["count"], cid + " (compiler's own restrictions)"
+        assert stm.count(G, plan2, stm.stm_tuning_default(jit=1)) == d["count"], cid + " (specialised kernel)"
+        assert stm.stm_last_launch()["jit"] == 1
 
 
 def stratified_roots(n, sizes, seed=5):
@@ -229,8 +231,8 @@ def test_config_scale_sampled_roots(cfg, name, sizes):
     p = CATALOG[name]
     plan = stm.Plan(p.k, p.edges)
     R = oracle.gk_restrictions(p.k, p.edges)
-    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default())
-    assert stm.stm_last_launch()["ranked"] == 1
+    tot, pr = stm.stm_match_count_per_root(G.handle, plan.handle, stm.stm_tuning_default(jit=1))
+    assert stm.stm_last_launch()["ranked"] == 1 and stm.stm_last_launch()["jit"] == 1
     assert int(pr.sum(dtype=np.uint64)) == tot
     rank2orig, gr = degree_ranked(g)
     roots = stratified_roots(g.n, sizes)
