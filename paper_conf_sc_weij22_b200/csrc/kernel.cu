@@ -98,6 +98,12 @@
 #else
 #define STM_SYM(x) x
 #endif
+#ifndef STM_ELEM_NOINLINE
+#define STM_ELEM_NOINLINE 1 // 1: run_jobs' element loop is one out-of-line function (i-cache)
+#endif
+#ifndef STM_ELEM_INLINE_MAX
+#define STM_ELEM_INLINE_MAX 0  // element streams up to this long run the inline copy instead
+#endif
 #ifndef STM_CPLAN
 #define STM_CPLAN 0         // 1: plan-specialised build: the plan is the compile-time record of
 #endif                      //    STM_CPLAN_HEADER (tools/cplan.py) instead of kp.plan
@@ -490,6 +496,84 @@ __device__ __forceinline__ void row_narrow(const W& w, int v, const int*& p, int
 
 __device__ __forceinline__ int log2c(int n) { return 32 - __clz(n); }  // ceil(log2(n+1))
 
+struct ElemOut {
+  unsigned long long jc;
+  int outc;
+};
+
+// The element loop of a combined set operation (Fig. 8): 32 elements of the flattened
+// job stream per pass -- per-lane job lookup, membership probe, ballot compaction into
+// the output set (materialise) or a popcount (count).  Out of line so that every
+// run_jobs call site shares one copy (measured: i-cache stalls).
+__device__ __forceinline__ ElemOut elem_loop_inl(const int lane, const int incl, const int total, const int start,
+                                          const unsigned long long Dll, const unsigned long long Pll,
+                                          const unsigned long long Oll, const int plen, const int flags,
+                                          const int lo, const int hi, const unsigned lab, const bool mine,
+                                          const bool count_mode, const uint8_t* const glabels,
+                                          const unsigned char* const l2s) {
+  int outc = 0;
+  unsigned long long jc = 0;
+  for (int e0 = 0; e0 < total; e0 += 32) {
+    const int e = e0 + lane;
+    int j = 0;
+#pragma unroll
+    for (int step = 16; step > 0; step >>= 1) {
+      int v = __shfl_sync(FULLMASK, incl, j + step - 1);
+      if (v <= e) j += step;
+    }
+    const bool valid = e < total;
+    const int* Dj = (const int*)__shfl_sync(FULLMASK, Dll, j);
+    const int* Pj = (const int*)__shfl_sync(FULLMASK, Pll, j);
+    const int sj = __shfl_sync(FULLMASK, start, j);
+    const int pl = __shfl_sync(FULLMASK, plen, j);
+    const int fj = __shfl_sync(FULLMASK, flags, j);
+    const int loj = __shfl_sync(FULLMASK, lo, j);
+    const int hij = __shfl_sync(FULLMASK, hi, j);
+    const unsigned labj = __shfl_sync(FULLMASK, lab, j);
+    bool keep = false;
+    int x = 0;
+    if (valid) {
+      x = Dj[e - sj];
+      keep = x > loj && x < hij;
+      if (keep && (fj & 1)) {
+        bool f;
+        if (fj & 8) f = (__ldg((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
+        else f = member(Pj, pl, x);
+        keep = (fj & 4) ? !f : f;
+      }
+      if (keep && labj != STM_LAB_ANY) keep = (l2s[glabels[x]] & labj) != 0;
+    }
+    const unsigned km = __ballot_sync(FULLMASK, keep);
+    // lanes of my own job inside this chunk
+    int a = start - e0, b = incl - e0;
+    a = a < 0 ? 0 : a;
+    b = b > 32 ? 32 : b;
+    unsigned rmask = 0;
+    if (mine && a < b) rmask = (b == 32 ? FULLMASK : ((1u << b) - 1)) & ~((1u << a) - 1);
+    if (count_mode) {
+      jc += __popc(km & rmask);
+    } else {
+      int* Oj = (int*)__shfl_sync(FULLMASK, Oll, j);
+      int base = __shfl_sync(FULLMASK, outc, j);
+      int fl = sj - e0;
+      fl = fl < 0 ? 0 : fl;
+      unsigned before = km & ((1u << lane) - 1) & ~((1u << fl) - 1);
+      if (keep) Oj[base + __popc(before)] = x;
+      outc += __popc(km & rmask);
+    }
+  }
+  return ElemOut{jc, outc};
+}
+__device__ __noinline__ ElemOut elem_loop(const int lane, const int incl, const int total, const int start,
+                                          const unsigned long long Dll, const unsigned long long Pll,
+                                          const unsigned long long Oll, const int plen, const int flags,
+                                          const int lo, const int hi, const unsigned lab, const bool mine,
+                                          const bool count_mode, const uint8_t* const glabels,
+                                          const unsigned char* const l2s) {
+  return elem_loop_inl(lane, incl, total, start, Dll, Pll, Oll, plen, flags, lo, hi, lab, mine, count_mode,
+                       glabels, l2s);
+}
+
 // Returns the (warp-uniform) number of kept elements summed over all jobs when
 // counting; in materialise mode *outc (lane j) receives job j's output size.  probe:
 // count mode for the candidate-set pre-test (plan.h pretest) -- *outc (lane j) receives
@@ -558,6 +642,26 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
   const int flags = (Pp != nullptr ? 1 : 0) | (J.op == STM_OP_DIFF ? 4 : 0) | (pslot >= 0 ? 8 : 0);
   const uint8_t* const glabels = w.kp->labels;
   const unsigned char* const l2s = w.bh->lab2slot;
+#if STM_ELEM_NOINLINE && !STM_LIST
+  // one out-of-line copy of the element loop for every call site (i-cache: the plan-
+  // specialised kernels instantiate run_jobs once per frame and kind); short streams stay
+  // inline (the call costs more than it saves there)
+  unsigned long long jc = jc0;
+  int outc = 0;
+  if (total > STM_ELEM_INLINE_MAX) {
+    const ElemOut eo = elem_loop(lane, incl, total, start, (unsigned long long)D, (unsigned long long)Pp,
+                                 (unsigned long long)J.out, plen, flags, J.lo, J.hi, J.lab, mine, count_mode,
+                                 glabels, l2s);
+    jc += eo.jc;
+    outc = eo.outc;
+  } else {
+    const ElemOut eo = elem_loop_inl(lane, incl, total, start, (unsigned long long)D, (unsigned long long)Pp,
+                                     (unsigned long long)J.out, plen, flags, J.lo, J.hi, J.lab, mine, count_mode,
+                                     glabels, l2s);
+    jc += eo.jc;
+    outc = eo.outc;
+  }
+#else
   int outc = 0;
   unsigned long long jc = jc0;
   const unsigned long long Dll = (unsigned long long)D, Pll = (unsigned long long)Pp,
@@ -642,6 +746,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       outc += __popc(km & rmask);
     }
   }
+#endif
   PROF_END(11, total)
   if (probe) {
     *outc_lane = (int)jc;
