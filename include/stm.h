@@ -183,8 +183,8 @@ typedef struct stm_tuning {
                              (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
                              than half the L2.  Speed only.  Default 0. */
   int32_t root_order;     /* order in which root chunks are handed out: 1 = ascending vertex id,
-                             2 = descending (heavy roots first on the degree-ranked copy); 0 = auto
-                             (ascending: descending measured slower on C2/C3).  Speed only. */
+                             2 = descending (heavy roots first on the degree-ranked copy), 3 = work-
+                             balanced chunks interleaved light / heavy; 0 = auto (ascending).  Speed only. */
   int32_t l2_persist_mb;  /* L2 persisting access-policy window over the longest neighbour lists (the
                              tail of the degree-ranked col_idx) when the CSR does not fit in half the L2:
                              0 = auto (off: measured no gain on C5), -1 = off, else MiB (capped by the

@@ -1515,7 +1515,8 @@ __device__ __noinline__ bool try_chunk(const StmKParams& kp) {
       long long c = (long long)r + (long long)kp.world * (long long)idx;
       if (kp.chunk_bounds) {  // work-balanced chunks (positions [bounds[c], bounds[c+1]))
         if (c < kp.n_chunks) {
-          if (kp.root_desc) c = kp.n_chunks - 1 - c;  // the heaviest (last) chunks first
+          if (kp.root_desc == 1) c = kp.n_chunks - 1 - c;  // the heaviest (last) chunks first
+          else if (kp.root_desc == 2) c = (c & 1) ? kp.n_chunks - 1 - (c >> 1) : (c >> 1);  // interleaved
           from = r;
           b = __ldg(&kp.chunk_bounds[c]);
           e = __ldg(&kp.chunk_bounds[c + 1]);
@@ -1529,7 +1530,7 @@ __device__ __noinline__ bool try_chunk(const StmKParams& kp) {
         from = r;
         b = (int)rb;
         e = (int)min((long long)kp.n, rb + kp.chunk);
-        if (kp.root_desc) {  // chunk c covers [lo + n - e, lo + n - b): the highest ids first
+        if (kp.root_desc == 1) {  // chunk c covers [lo + n - e, lo + n - b): the highest ids first
           const int nb = (int)(kp.root_lo + kp.n - e);
           e = (int)(kp.root_lo + kp.n - b);
           b = nb;

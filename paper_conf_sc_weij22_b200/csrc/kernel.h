@@ -129,7 +129,8 @@ struct StmKParams {
   const int32_t* root_map;        // counting id -> caller's id (degree-ranked copy), or NULL
   unsigned long long* cursors[8]; // chunk cursors (own rank + optional peers)
   int32_t rank, world, chunk;
-  int32_t root_desc;              // 1: chunk c covers the root ids [n-(c+1)chunk, n-c*chunk) (descending)
+  int32_t root_desc;              // 1: chunk c covers the root ids [n-(c+1)chunk, n-c*chunk) (descending);
+                                  // 2: work-balanced chunks interleaved light / heavy (c even: c/2, odd: from the end)
   int32_t local_steal, global_steal, stop_level, detect_level, unroll, root_batch;
   int32_t count_bytes;            // 1 = accumulate algorithmic bytes (instrumented launch)
   int32_t ht_slots;               // per-warp shared-memory hash slots (0 = off)

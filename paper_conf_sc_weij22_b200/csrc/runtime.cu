@@ -760,7 +760,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (tin) t = *tin; else stm_tuning_default(&t);
   if (t.unroll < 0 || t.unroll > STM_UMAX) return stm_fail(STM_EINVAL, "unroll %d not in 0..%d", t.unroll, STM_UMAX);
   if (t.occupancy < 0 || t.occupancy > 2) return stm_fail(STM_EINVAL, "occupancy %d not in 0..2", t.occupancy);
-  if (t.root_order < 0 || t.root_order > 2) return stm_fail(STM_EINVAL, "root_order %d not in 0..2", t.root_order);
+  if (t.root_order < 0 || t.root_order > 3) return stm_fail(STM_EINVAL, "root_order %d not in 0..3", t.root_order);
   if (t.root_chunk < 0) return stm_fail(STM_EINVAL, "root_chunk %d < 0", t.root_chunk);
   if (t.block_warps == 0) t.block_warps = 16;
   if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
@@ -863,7 +863,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   const int root_chunk = t.root_chunk ? t.root_chunk : (variant == 2 ? 2 : 1);
   // root order: ascending by default -- descending (high-degree roots first on the
   // ranked copy) measured 1.2-1.7x slower on C2/C3 and neutral on C5
-  kp.root_desc = t.root_order == 2 ? 1 : 0;
+  kp.root_desc = t.root_order == 2 ? 1 : t.root_order == 3 ? 2 : 0;
   // L2 persistence (B200 126 MB L2): on the degree-ranked copy the rows are in degree
   // order, so the tail of col_idx holds the longest lists -- the ones every set
   // operation probes.  Keep up to l2_persist_mb of it persisting in L2 when the CSR
@@ -918,7 +918,10 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (oe != 0) return stm_fail(STM_ECUDA, "occupancy (variant %d, %s build, %d warps): %s", variant, la ? "list" : t.instrument ? "instr" : "count", t.block_warps, cudaGetErrorString((cudaError_t)oe));
   if (bps < 1) return stm_fail(STM_EUNSUPPORTED, "kernel does not fit on an SM with %d warps", t.block_warps);
   if (t.blocks_per_sm > 0) bps = std::min(bps, t.blocks_per_sm);
-  const int grid = bps * g->num_sms;
+  // no more warps than root chunks (tiny graphs: the idle surplus would only add start-up,
+  // work-sharing and termination traffic)
+  int grid = bps * g->num_sms;
+  if (kp.chunk_bounds && !shard) grid = (int)std::max<int64_t>(1, std::min<int64_t>(grid, (kp.n_chunks + t.block_warps - 1) / t.block_warps));
   const int64_t warps = (int64_t)grid * t.block_warps;
   const size_t arena_bytes = (size_t)warps * (size_t)P.n_nodes * (size_t)kp.cap * sizeof(int32_t);
   // task pool: never more tasks than blocks (StmWork::deficit), capacity 2 * grid rounded up

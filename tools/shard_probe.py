@@ -14,20 +14,21 @@ from paper_conf_sc_weij22_b200 import stm  # noqa: E402
 
 cfg, pats = sys.argv[1], sys.argv[2].split(",")
 tk = dict(a.split("=") for a in sys.argv[3:] if "=" in a)
+WS = tuple(int(x) for x in tk.pop("ws", "1,2,4,8").split(","))
 g = stmgen.config_graph(cfg)
 G = stm.Graph.from_stmgen(g)
 t = stm.stm_tuning_default(**{k: int(v) for k, v in tk.items()})
-cur = torch.zeros(64, dtype=torch.int64, device="cuda")
+cur = torch.zeros(64 * max(WS), dtype=torch.int64, device="cuda")
 for name in pats:
     p = stmgen.CATALOG[name]
     plan = stm.Plan(p.k, p.edges, None)
     total = None
     t1 = None
-    for W in (1, 2, 4, 8):
+    for W in WS:
         times, cnt = [], 0
         for r in range(W):
             ptrs = [None] * 8
-            ptrs[r] = cur.data_ptr() + 64 * r
+            ptrs[r] = cur.data_ptr() + 64 * r  # own cursor only (no cross-GPU stealing)
             sh = stm.make_shard(r, W, 0, ptrs)  # chunk 0: the launch's root_chunk (as dist.py)
             best = 1e9
             for _ in range(2):
