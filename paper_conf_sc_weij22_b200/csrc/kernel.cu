@@ -101,6 +101,9 @@
 #ifndef STM_ELEM_NOINLINE
 #define STM_ELEM_NOINLINE 1 // 1: run_jobs' element loop is one out-of-line function (i-cache)
 #endif
+#ifndef STM_GCHK_CYCLES
+#define STM_GCHK_CYCLES 4096  // busy warps look at the pool's demand at most this often (SM cycles)
+#endif
 #ifndef STM_ELEM_INLINE_MAX
 #define STM_ELEM_INLINE_MAX 0  // element streams up to this long run the inline copy instead
 #endif
@@ -850,13 +853,13 @@ __device__ __forceinline__ int waiting_warps(const W& w) {
   if (w.lane == 0) m = *(volatile int*)&w.bh->idle_mask;
   return __shfl_sync(FULLMASK, m, 0);
 }
-// Grid status, looked at (two L2 loads) at most every ~0.5 us per warp: does the pool want
+// Grid status, looked at (two L2 loads) at most every ~2 us per warp: does the pool want
 // a task (block pollers waiting)?  Is the grid starving (WarpHdr::deep, split_stop)?
 __device__ __forceinline__ bool pool_wanted(const W& w) {
   int want = 0;
   if (w.lane == 0) {
     const long long now = clock64();
-    if (now - w.h->gchk >= 1024) {
+    if (now - w.h->gchk >= STM_GCHK_CYCLES) {
       w.h->gchk = now;
       volatile StmWork* vw = w.kp->work;
       want = vw->deficit > 0;
