@@ -101,6 +101,17 @@
 #ifndef STM_ELEM_NOINLINE
 #define STM_ELEM_NOINLINE 1 // 1: run_jobs' element loop is one out-of-line function (i-cache)
 #endif
+#ifndef STM_BM_CS
+#define STM_BM_CS 1         // 1: hub-bitmap probes as streaming loads (L2 evict-first; K6-e -3 %)
+#endif
+#if STM_BM_CS
+#define STM_BM_LOAD(p) __ldcs(p)
+#else
+#define STM_BM_LOAD(p) __ldg(p)
+#endif
+#ifndef STM_BATCH_ELEMS
+#define STM_BATCH_ELEMS 0   // > 0: admit siblings into a batch only while the summed set-size
+#endif                      //    bounds stay within this many elements (0: the arena region)
 #ifndef STM_GCHK_CYCLES
 #define STM_GCHK_CYCLES 4096  // busy warps look at the pool's demand at most this often (SM cycles)
 #endif
@@ -540,7 +551,7 @@ __device__ __forceinline__ ElemOut elem_loop_inl(const int lane, const int incl,
       keep = x > loj && x < hij;
       if (keep && (fj & 1)) {
         bool f;
-        if (fj & 8) f = (__ldg((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
+        if (fj & 8) f = (STM_BM_LOAD((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
         else f = member(Pj, pl, x);
         keep = (fj & 4) ? !f : f;
       }
@@ -693,7 +704,7 @@ __device__ JOBS_INL unsigned long long run_jobs(W& w, Job J, int njobs, bool cou
       keep = x > loj && x < hij;
       if (keep && (fj & 1)) {
         bool f;
-        if (fj & 8) f = (__ldg((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
+        if (fj & 8) f = (STM_BM_LOAD((const unsigned*)Pj + (x >> 5)) >> (x & 31)) & 1u;
         else f = member(Pj, pl, x);
         keep = (fj & 4) ? !f : f;
       }
@@ -1190,7 +1201,9 @@ __device__ GATHER_SLOW_INL int gather_batch_slow(W& w, int F, int U, const int* 
         int t = __shfl_up_sync(FULLMASK, inc, o);
         if (w.lane >= o) inc += t;
       }
-      if (pass && w.h->used[s - nb] + inc > cap) fits = false;
+      // (the first candidate of a batch is always admitted: its bound fits the region, and the
+      // batch budget STM_BATCH_ELEMS only limits how many more join it)
+      if (pass && w.h->used[s - nb] + inc > cap && !(m == 0 && inc == ub)) fits = false;
     }
     unsigned pm = __ballot_sync(FULLMASK, pass);
     unsigned fm = __ballot_sync(FULLMASK, pass && fits);
@@ -1258,8 +1271,12 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
   // Fast admission: when U copies of every node's candidate-independent size bound
   // fit in its region, any batch of <= U candidates fits -- fixed slice offsets
   // t * bound, no per-candidate degree loads or prefix sums.
+  // batch budget: the sets of one batch are built by one combined operation that is never
+  // split by work sharing, so it is kept to about STM_BATCH_ELEMS driving elements (not the
+  // whole arena region) -- heavy hub siblings then stay in the frame, stealable
+  const int capb = STM_BATCH_ELEMS > 0 ? min(cap, STM_BATCH_ELEMS) : cap;
   bool fixed = true;
-  for (int s = nb; s < ne && fixed; ++s) fixed = (long long)node_ub_const(w, s, F, u) * U <= (long long)cap;
+  for (int s = nb; s < ne && fixed; ++s) fixed = (long long)node_ub_const(w, s, F, u) * U <= (long long)capb;
   if (fixed) {
     int m = 0;
     while (m < U && pos < e) {
@@ -1289,7 +1306,7 @@ __device__ STEP_INL int gather_batch(W& w, int F, int U) {
     __syncwarp();
     return m;
   }
-  return gather_batch_slow(w, F, U, src, lo, hi, pos, e, nb, ne, cap, u);
+  return gather_batch_slow(w, F, U, src, lo, hi, pos, e, nb, ne, capb, u);
 }
 
 // root batch: up to root_batch roots from [root_it, root_end) with the root label

@@ -391,8 +391,14 @@ extern "C" stm_status stm_motif_census(const stm_graph* g, int k, uint32_t flags
   int launches = 0;
   stm_status s = STM_OK;
   if (per_motif || k < 3) {  // one counting launch per motif (A/B baseline; k = 2 has one motif)
+    // the generic kernel unless specialised kernels are asked for explicitly (one NVRTC
+    // compile per motif would dominate the census)
+    stm_tuning tt;
+    if (t) tt = *t;
+    else stm_tuning_default(&tt);
+    if (tt.jit != 1) tt.jit = -1;
     for (size_t i = 0; i < cat.size() && s == STM_OK; ++i) {
-      s = stm_match_count_ex(g, plans[i], t, nullptr, stream, &out[i]);
+      s = stm_match_count_ex(g, plans[i], &tt, nullptr, stream, &out[i]);
       ++launches;
     }
   } else {
