@@ -59,6 +59,10 @@ def _load():
         lib.oracle_count.argtypes = [ctypes.c_int64, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp, vp,
                                      ctypes.c_int, ctypes.c_int, vp, ctypes.c_int, vp, ctypes.c_int64,
                                      ctypes.c_int, vp, ctypes.POINTER(ctypes.c_uint64)]
+        lib.oracle_count_directed.restype = ctypes.c_int
+        lib.oracle_count_directed.argtypes = [ctypes.c_int64, vp, vp, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp,
+                                              vp, ctypes.c_int, ctypes.c_int, vp, ctypes.c_int, vp,
+                                              ctypes.c_int64, ctypes.c_int, vp, ctypes.POINTER(ctypes.c_uint64)]
         lib.oracle_list.restype = ctypes.c_int
         lib.oracle_list.argtypes = [ctypes.c_int64, vp, vp, vp, ctypes.c_int, ctypes.c_int, vp, vp,
                                     ctypes.c_int, ctypes.c_int, vp, ctypes.c_int, vp, ctypes.c_int64,
@@ -139,6 +143,94 @@ def list_embeddings(g, k: int, edges: Sequence[Tuple[int, int]], plabels: Option
         raise ValueError("oracle_list rejected its input")
     got = buf[:min(int(nl.value), int(capacity))]
     return got[np.lexsort(got.T[::-1])] if got.shape[0] else got
+
+
+def transpose(n: int, row_ptr: np.ndarray, col_idx: np.ndarray):
+    """In-neighbour rows of a digraph given by its out-neighbour rows (sorted ascending)."""
+    rp = np.asarray(row_ptr, dtype=np.int64)
+    ci = np.asarray(col_idx, dtype=np.int64)
+    src = np.repeat(np.arange(n, dtype=np.int64), np.diff(rp))
+    o = np.lexsort((src, ci))  # by destination, then source
+    in_rp = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(ci, minlength=n), out=in_rp[1:])
+    return in_rp, np.ascontiguousarray(src[o], dtype=np.int32)
+
+
+def count_directed(g, k: int, arcs: Sequence[Tuple[int, int]], plabels: Optional[Sequence[int]] = None,
+                   vertex_induced: bool = False, restrictions: Sequence[Tuple[int, int]] = (),
+                   root_u: int = -1, roots: Optional[np.ndarray] = None, threads: int = 0,
+                   per_root: bool = False):
+    """count() for a directed data graph (g.row_ptr / g.col_idx = sorted out-neighbour rows)
+    and a pattern given by arcs (a, b) = a -> b (oracle.c oracle_count_directed)."""
+    lib = _load()
+    rp = np.ascontiguousarray(g.row_ptr, dtype=np.int64)
+    ci = np.ascontiguousarray(g.col_idx, dtype=np.int32)
+    irp, ici = transpose(g.n, rp, ci)
+    lab = None
+    if plabels is not None:
+        if g.labels is None:
+            raise ValueError("labeled pattern on an unlabeled graph")
+        lab = np.ascontiguousarray(g.labels, dtype=np.int32)
+    e = np.ascontiguousarray(np.asarray(arcs, dtype=np.int32).reshape(-1, 2))
+    pl = None if plabels is None else np.ascontiguousarray(np.asarray(plabels, dtype=np.int32))
+    r = np.ascontiguousarray(np.asarray(restrictions, dtype=np.int32).reshape(-1, 2))
+    ro = None if roots is None else np.ascontiguousarray(np.asarray(roots, dtype=np.int64))
+    nr = 0 if ro is None else ro.shape[0]
+    pr = np.zeros(nr if ro is not None else g.n, dtype=np.uint64) if per_root else None
+    out = ctypes.c_uint64(0)
+    rc = lib.oracle_count_directed(g.n, _ptr(rp), _ptr(ci), _ptr(irp), _ptr(ici), _ptr(lab), k, e.shape[0],
+                                   _ptr(e), _ptr(pl), int(vertex_induced), r.shape[0], _ptr(r), root_u,
+                                   _ptr(ro), nr, threads or (os.cpu_count() or 1), _ptr(pr), ctypes.byref(out))
+    if rc != 0:
+        raise ValueError("oracle_count_directed rejected its input")
+    return (int(out.value), pr) if per_root else int(out.value)
+
+
+def brute_force_count_directed(g, k: int, arcs, plabels=None, vertex_induced=False, restrictions=()) -> int:
+    """The directed definition tested literally on every injective map f: V_Q -> V: every
+    pattern arc a -> b an arc f(a) -> f(b) of g, [vertex-induced] every pattern non-arc a
+    non-arc.  Tiny graphs only."""
+    A = _adj_sets(g)
+    E = {(a, b) for a, b in arcs}
+    non = [(a, b) for a in range(k) for b in range(k) if a != b and (a, b) not in E]
+    c = 0
+    for f in itertools.permutations(range(g.n), k):
+        if any(f[b] not in A[f[a]] for a, b in E):
+            continue
+        if vertex_induced and any(f[b] in A[f[a]] for a, b in non):
+            continue
+        if plabels is not None and any(int(g.labels[f[u]]) != int(plabels[u]) for u in range(k)):
+            continue
+        if any(not f[a] < f[b] for a, b in restrictions):
+            continue
+        c += 1
+    return c % (1 << 64)
+
+
+def automorphisms_directed(k: int, arcs, plabels=None) -> List[Tuple[int, ...]]:
+    """All label- and arc-preserving permutations of a directed pattern (brute force)."""
+    E = {(a, b) for a, b in arcs}
+    out = []
+    for p in itertools.permutations(range(k)):
+        if plabels is not None and any(plabels[p[u]] != plabels[u] for u in range(k)):
+            continue
+        if all((p[a], p[b]) in E for a, b in E):
+            out.append(p)
+    return out
+
+
+def gk_restrictions_directed(k: int, arcs, plabels=None) -> List[Tuple[int, int]]:
+    """gk_restrictions over the automorphism group of a directed pattern."""
+    group = automorphisms_directed(k, arcs, plabels)
+    R: List[Tuple[int, int]] = []
+    while len(group) > 1:
+        for u in range(k):
+            orbit = sorted({p[u] for p in group})
+            if len(orbit) > 1:
+                break
+        R.extend((u, w) for w in orbit if w != u)
+        group = [p for p in group if p[u] == u]
+    return R
 
 
 # ---------------------------------------------------------------- brute force

@@ -32,6 +32,18 @@
  *
  * Input requirements: undirected simple graph, rows sorted ascending (checked
  * by the Python wrapper), pattern connected with 1 <= k <= 16.
+ *
+ * Directed graphs ("supports both directed and undirected graphs";
+ * SURVEY.md 8(f) NEXT-4), oracle_count_directed: G is a simple digraph given by its
+ * sorted out-neighbour rows (and, for candidate generation only, the transposed in-
+ * neighbour rows); Q's edges are ordered pairs (a, b) = arc a -> b.  The definition is
+ * the same with arcs:
+ *
+ *   for every pattern arc a -> b:                f(a) -> f(b) is an arc of G
+ *   [vertex-induced] every pattern non-arc a -> b: f(a) -> f(b) is not an arc of G
+ *
+ * checked literally per candidate (arc x -> y = y in out(x), binary search); the
+ * matching order is the BFS over Q's underlying undirected graph.
  */
 #include <pthread.h>
 #include <stdatomic.h>
@@ -67,6 +79,12 @@ typedef struct {
   int32_t *list;
   uint64_t list_cap;
   atomic_ullong list_n;
+  /* directed graphs: dadj[a][b] = 1 iff pattern arc a -> b; adj is then its underlying
+     undirected graph (BFS order only); in_* = transposed rows (candidates only) */
+  int directed;
+  int dadj[OMAX][OMAX];
+  const int64_t *in_row_ptr;
+  const int32_t *in_col_idx;
 } ojob;
 
 typedef struct {
@@ -108,6 +126,66 @@ static int consistent(const ostate *S, int l, int u, int64_t w) {
     if ((a == u || b == u) && fa >= 0 && fb >= 0 && !(fa < fb)) return 0;
   }
   return 1;
+}
+
+/* directed: the definition with arcs, checked literally (arc x -> y: y in out(x)) */
+static int consistent_directed(const ostate *S, int l, int u, int64_t w) {
+  const ojob *J = S->J;
+  if (J->use_labels && J->labels[w] != J->plabel[u]) return 0;
+  for (int j = 0; j < l; ++j) {
+    int q = J->order[j];
+    int64_t fq = S->f[q];
+    if (fq == w) return 0; /* injective */
+    if (J->dadj[q][u]) {
+      if (!adjacent(J, fq, w)) return 0; /* pattern arc q -> u must be a data arc */
+    } else if (J->vertex_induced) {
+      if (adjacent(J, fq, w)) return 0;
+    }
+    if (J->dadj[u][q]) {
+      if (!adjacent(J, w, fq)) return 0; /* pattern arc u -> q must be a data arc */
+    } else if (J->vertex_induced) {
+      if (adjacent(J, w, fq)) return 0;
+    }
+  }
+  for (int r = 0; r < J->n_restr; ++r) {
+    int a = J->restr[2 * r], b = J->restr[2 * r + 1];
+    int64_t fa = (a == u) ? w : S->f[a];
+    int64_t fb = (b == u) ? w : S->f[b];
+    if ((a == u || b == u) && fa >= 0 && fb >= 0 && !(fa < fb)) return 0;
+  }
+  return 1;
+}
+
+static void rec_directed(ostate *S, int l) {
+  const ojob *J = S->J;
+  if (l == J->k) {
+    S->count += 1;
+    return;
+  }
+  int u = J->order[l];
+  /* candidates: the out-row of f(q) for a pattern arc q -> u, or the in-row of f(q) for
+     u -> q, whichever matched pattern neighbour gives the shortest row */
+  const int32_t *best = NULL;
+  int64_t bestlen = -1;
+  for (int j = 0; j < l; ++j) {
+    int q = J->order[j];
+    int64_t fq = S->f[q];
+    if (J->dadj[q][u]) {
+      int64_t d = J->row_ptr[fq + 1] - J->row_ptr[fq];
+      if (bestlen < 0 || d < bestlen) { best = J->col_idx + J->row_ptr[fq]; bestlen = d; }
+    }
+    if (J->dadj[u][q]) {
+      int64_t d = J->in_row_ptr[fq + 1] - J->in_row_ptr[fq];
+      if (bestlen < 0 || d < bestlen) { best = J->in_col_idx + J->in_row_ptr[fq]; bestlen = d; }
+    }
+  }
+  for (int64_t e = 0; e < bestlen; ++e) {
+    int64_t w = best[e];
+    if (!consistent_directed(S, l, u, w)) continue;
+    S->f[u] = w;
+    rec_directed(S, l + 1);
+    S->f[u] = -1;
+  }
 }
 
 static void rec(ostate *S, int l) {
@@ -152,7 +230,13 @@ static void *worker(void *arg) {
       uint64_t before = S->count;
       int u0 = J->order[0];
       for (int x = 0; x < OMAX; ++x) S->f[x] = -1;
-      if (consistent(S, 0, u0, v)) {
+      if (J->directed) {
+        if (consistent_directed(S, 0, u0, v)) {
+          S->f[u0] = v;
+          rec_directed(S, 1);
+          S->f[u0] = -1;
+        }
+      } else if (consistent(S, 0, u0, v)) {
         S->f[u0] = v;
         rec(S, 1);
         S->f[u0] = -1;
@@ -200,15 +284,21 @@ static int run(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const 
                int k, int n_edges, const int32_t *edges, const int32_t *plabels,
                int vertex_induced, int n_restr, const int32_t *restr, int root_u,
                const int64_t *roots, int64_t n_roots, int nthreads, uint64_t *per_root,
-               int32_t *list, uint64_t list_cap, uint64_t *list_n, uint64_t *out_count) {
+               int32_t *list, uint64_t list_cap, uint64_t *list_n, uint64_t *out_count,
+               const int64_t *in_row_ptr, const int32_t *in_col_idx) {
   if (k < 1 || k > OMAX) return -1;
   ojob *J = (ojob *)calloc(1, sizeof(ojob));
   J->n = n; J->row_ptr = row_ptr; J->col_idx = col_idx; J->labels = labels;
   J->k = k;
+  J->directed = in_row_ptr != NULL;
+  J->in_row_ptr = in_row_ptr;
+  J->in_col_idx = in_col_idx;
+  if (J->directed && list) { free(J); return -1; }
   for (int i = 0; i < n_edges; ++i) {
     int a = edges[2 * i], b = edges[2 * i + 1];
     if (a < 0 || b < 0 || a >= k || b >= k || a == b) { free(J); return -1; }
     J->adj[a][b] = J->adj[b][a] = 1;
+    J->dadj[a][b] = 1;
   }
   if (root_u >= k) { free(J); return -1; }
   if (!bfs_order(k, J->adj, root_u, J->order)) { free(J); return -1; }
@@ -258,7 +348,18 @@ int oracle_count(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, cons
                  const int64_t *roots, int64_t n_roots, int nthreads, uint64_t *per_root,
                  uint64_t *out_count) {
   return run(n, row_ptr, col_idx, labels, k, n_edges, edges, plabels, vertex_induced, n_restr, restr, root_u,
-             roots, n_roots, nthreads, per_root, NULL, 0, NULL, out_count);
+             roots, n_roots, nthreads, per_root, NULL, 0, NULL, out_count, NULL, NULL);
+}
+
+/* directed graphs: `edges` are arcs (a -> b); in_row_ptr / in_col_idx = the transposed rows */
+int oracle_count_directed(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int64_t *in_row_ptr,
+                          const int32_t *in_col_idx, const int32_t *labels, int k, int n_edges,
+                          const int32_t *edges, const int32_t *plabels, int vertex_induced, int n_restr,
+                          const int32_t *restr, int root_u, const int64_t *roots, int64_t n_roots,
+                          int nthreads, uint64_t *per_root, uint64_t *out_count) {
+  if (!in_row_ptr || !in_col_idx) return -1;
+  return run(n, row_ptr, col_idx, labels, k, n_edges, edges, plabels, vertex_induced, n_restr, restr, root_u,
+             roots, n_roots, nthreads, per_root, NULL, 0, NULL, out_count, in_row_ptr, in_col_idx);
 }
 
 /* count and list: list[i*k + u] = f(u) for the first min(count, list_cap) embeddings found
@@ -269,5 +370,5 @@ int oracle_list(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const
                 const int64_t *roots, int64_t n_roots, int nthreads,
                 int32_t *list, uint64_t list_cap, uint64_t *list_n, uint64_t *out_count) {
   return run(n, row_ptr, col_idx, labels, k, n_edges, edges, plabels, vertex_induced, n_restr, restr, root_u,
-             roots, n_roots, nthreads, NULL, list, list_cap, list_n, out_count);
+             roots, n_roots, nthreads, NULL, list, list_cap, list_n, out_count, NULL, NULL);
 }
