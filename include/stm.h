@@ -65,10 +65,13 @@ enum {
   STM_AUTO_ORDER = 8,      /* ignore `order`; use the greedy connected order */
   STM_CENSUS_PER_MOTIF = 32, /* stm_motif_census only: one counting launch per motif instead of the merged
                                 trie launch (A/B baseline of pattern merging) */
-  STM_LAZY_UNBOUNDED = 16  /* code motion hoists only set chains that carry a restriction bound for their
+  STM_LAZY_UNBOUNDED = 16, /* code motion hoists only set chains that carry a restriction bound for their
                               consumer; a chain unbounded at its first operation is computed at the level
                               of its first consumer (no hoisting across levels whose prefixes rarely extend;
                               speed only) */
+  STM_DIRECTED = 64        /* directed pattern (NEXT-4): `edges` are arcs (a, b) = a -> b, and
+                              the plan counts in graphs loaded with stm_graph_load_directed: every arc of Q
+                              an arc of G (vertex-induced: every non-arc a non-arc) */
 };
 
 enum { STM_K_MAX = 8 };
@@ -105,6 +108,17 @@ stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_t* d_row_pt
 
 /* stm_graph_info -- n, number of directed adjacency entries (2m), max degree. Any out may be NULL. */
 stm_status stm_graph_info(const stm_graph* g, int64_t* n, int64_t* nnz, int64_t* max_degree);
+
+/*
+ * stm_graph_load_directed -- a directed simple graph (NEXT-4; "supports both directed
+ * and undirected graphs").  row_ptr / col_idx are the out-neighbour rows (arc v -> col_idx[e] for
+ * e in [row_ptr[v], row_ptr[v+1])), sorted strictly ascending, no self-loops, ids in [0, n); the
+ * in-rows are built here.  Both are device-resident (2 * m entries).  Counted with STM_DIRECTED
+ * plans only (STM_EINVAL otherwise).  No degree-ranked copy, hub bitmaps or root splitting (speed
+ * only).  Ownership, labels and errors as stm_graph_load.
+ */
+stm_status stm_graph_load_directed(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                                   const int32_t* labels, int device, stm_graph** out);
 
 stm_status stm_graph_free(stm_graph* g);
 

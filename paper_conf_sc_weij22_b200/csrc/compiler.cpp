@@ -54,8 +54,9 @@ static void build_describe(stm_plan* P) {
   const StmPlan& D = P->dev;
   std::string s;
   char buf[256];
-  snprintf(buf, sizeof buf, "k=%d mode=%s code_motion=%s count_mode=%s aut=%lld\n", D.k,
-           D.vertex_induced ? "vertex" : "edge", (P->flags & STM_NO_CODE_MOTION) ? "off" : "on",
+  snprintf(buf, sizeof buf, "k=%d mode=%s%s code_motion=%s count_mode=%s aut=%lld\n", D.k,
+           D.vertex_induced ? "vertex" : "edge", D.directed ? " directed" : "",
+           (P->flags & STM_NO_CODE_MOTION) ? "off" : "on",
            D.count_mode == STM_COUNT_FUSED ? "fused" : "frame", (long long)P->aut);
   s += buf;
   s += "order=[";
@@ -77,14 +78,18 @@ static void build_describe(stm_plan* P) {
       }
     return r + "}";
   };
+  auto rawn = [&](int code) -> std::string {  // position code j + 8 d (directed: d = 0 out-row, 1 in-row)
+    const std::string v = "(v" + std::to_string(code & 7) + ")";
+    return D.directed ? ((code >> 3) ? "N-" : "N+") + v : "N" + v;
+  };
   auto src = [&](const StmSrc& x) -> std::string {
-    return x.kind == STM_SRC_RAW ? "N(v" + std::to_string(x.idx) + ")" : "S" + std::to_string(x.idx);
+    return x.kind == STM_SRC_RAW ? rawn(x.idx) : "S" + std::to_string(x.idx);
   };
   for (int i = 0; i < D.n_nodes; ++i) {
     const StmNode& n = D.nodes[i];
-    std::string a = n.a_kind == STM_SRC_RAW ? "N(v" + std::to_string(n.a) + ")" : "S" + std::to_string(n.a);
-    snprintf(buf, sizeof buf, "S%d: level %d stage %d = %s %s N(v%d) lab=%s lo=%s hi=%s\n", i, n.level,
-             n.stage, a.c_str(), n.op == STM_OP_AND ? "&" : "-", n.b, lab(n.lab).c_str(),
+    std::string a = n.a_kind == STM_SRC_RAW ? rawn(n.a) : "S" + std::to_string(n.a);
+    snprintf(buf, sizeof buf, "S%d: level %d stage %d = %s %s %s lab=%s lo=%s hi=%s\n", i, n.level,
+             n.stage, a.c_str(), n.op == STM_OP_AND ? "&" : "-", rawn(n.b).c_str(), lab(n.lab).c_str(),
              fmt_mask(n.lo).c_str(), fmt_mask(n.hi).c_str());
     s += buf;
   }
@@ -97,8 +102,7 @@ static void build_describe(stm_plan* P) {
     s += buf;
   }
   const StmFilter& f = D.filt[D.k - 1];
-  std::string op = D.cnt_op == STM_OP_NONE ? "" : (D.cnt_op == STM_OP_AND ? " & N(v" : " - N(v") +
-                                                     std::to_string(D.cnt_b) + ")";
+  std::string op = D.cnt_op == STM_OP_NONE ? "" : (D.cnt_op == STM_OP_AND ? " & " : " - ") + rawn(D.cnt_b);
   if (D.cnt_op == STM_OP_NONE) op = "";
   snprintf(buf, sizeof buf, "count %d: %s%s lab=%s lo=%s hi=%s excl=%s\n", D.k - 1, src(D.cnt_a).c_str(),
            op.c_str(), lab(f.lab).c_str(), fmt_mask(f.lo).c_str(), fmt_mask(f.hi).c_str(),
@@ -121,18 +125,26 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   if (k < 2) return stm_fail(STM_EINVAL, "pattern size k=%d < 2 is not a matching query", k);
   if (k > STM_KMAX) return stm_fail(STM_EUNSUPPORTED, "pattern size k=%d > %d", k, STM_KMAX);
   if (n_edges < 1 || !edges) return stm_fail(STM_EINVAL, "pattern has no edges");
-  if (flags & ~0x1Fu) return stm_fail(STM_EINVAL, "unknown flag bits 0x%x", flags);
+  if (flags & ~(0x1Fu | STM_DIRECTED)) return stm_fail(STM_EINVAL, "unknown flag bits 0x%x", flags);
   const bool vi = flags & STM_VERTEX_INDUCED;
+  const bool directed = flags & STM_DIRECTED;  // edges are arcs a -> b (NEXT-4)
   const bool cm = !(flags & STM_NO_CODE_MOTION);
   const bool lazy = cm && (flags & STM_LAZY_UNBOUNDED);
 
-  int adj[STM_KMAX][STM_KMAX] = {};
+  int adj[STM_KMAX][STM_KMAX] = {};   // underlying undirected pattern graph
+  int dadj[STM_KMAX][STM_KMAX] = {};  // arcs (directed patterns; = adj for undirected ones)
   std::vector<std::pair<int, int>> E;
   for (int i = 0; i < n_edges; ++i) {
     int a = edges[2 * i], b = edges[2 * i + 1];
     if (a < 0 || b < 0 || a >= k || b >= k) return stm_fail(STM_EINVAL, "edge %d out of range", i);
     if (a == b) return stm_fail(STM_EINVAL, "self-loop in pattern at vertex %d", a);
-    if (!adj[a][b]) E.push_back({std::min(a, b), std::max(a, b)});
+    if (directed) {
+      if (!dadj[a][b]) E.push_back({a, b});
+      dadj[a][b] = 1;
+    } else {
+      if (!adj[a][b]) E.push_back({std::min(a, b), std::max(a, b)});
+      dadj[a][b] = dadj[b][a] = 1;
+    }
     adj[a][b] = adj[b][a] = 1;
   }
   {  // connectivity
@@ -161,9 +173,9 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     do {
       bool ok = true;
       for (int u = 0; u < k && ok; ++u) ok = lab[p[u]] == lab[u];
-      for (auto& e : E) {
+      for (auto& e : E) {  // (arcs map to arcs for directed patterns)
         if (!ok) break;
-        ok = adj[p[e.first]][p[e.second]];
+        ok = dadj[p[e.first]][p[e.second]];
       }
       if (ok) group.push_back(p);
     } while (next_perm(p));
@@ -267,6 +279,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   memset(&D, 0, sizeof D);
   D.k = k;
   D.vertex_induced = vi;
+  D.directed = directed ? 1 : 0;
   for (int l = 0; l < k; ++l) D.order[l] = pi[l];
 
   // label slots
@@ -281,12 +294,19 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     return 1u << (std::find(slots.begin(), slots.end(), x) - slots.begin());
   };
 
-  // per-position signatures, bounds, exclusions
-  int sig[STM_KMAX][STM_KMAX] = {};  // +1 adjacent, -1 difference (vertex-induced), 0 unconstrained
+  // per-position signatures, bounds, exclusions.  A raw operand is named by a position
+  // code j + 8 d: N(v_j) for undirected plans (d = 0); for directed ones d = 0 is the out-
+  // row N+(v_j) (pattern arc pi[j] -> pi[l]) and d = 1 the in-row N-(v_j) (arc pi[l] -> pi[j]).
+  int sig[STM_KMAX][2 * STM_KMAX] = {};  // per code: +1 member, -1 difference (vertex-induced), 0 none
   unsigned lo_pos[STM_KMAX] = {}, hi_pos[STM_KMAX] = {}, excl[STM_KMAX] = {};
   for (int l = 0; l < k; ++l)
     for (int j = 0; j < l; ++j) {
-      sig[l][j] = adj[pi[l]][pi[j]] ? 1 : (vi ? -1 : 0);
+      if (directed) {
+        sig[l][j] = dadj[pi[j]][pi[l]] ? 1 : (vi ? -1 : 0);
+        sig[l][j + 8] = dadj[pi[l]][pi[j]] ? 1 : (vi ? -1 : 0);
+      } else {
+        sig[l][j] = adj[pi[l]][pi[j]] ? 1 : (vi ? -1 : 0);
+      }
       if (less[pi[j]][pi[l]]) lo_pos[l] |= 1u << j;
       if (less[pi[l]][pi[j]]) hi_pos[l] |= 1u << j;
       if (!adj[pi[l]][pi[j]]) excl[l] |= 1u << j;
@@ -320,14 +340,21 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
   std::vector<StmSrc> cand_src(k);
   for (int l = 1; l < k; ++l) {
     Chain c;
-    for (int j = 0; j < l; ++j)
-      if (sig[l][j] == 1) { c.f = j; break; }
-    for (int j = 0; j < c.f; ++j)
-      if (sig[l][j] == -1) { c.ops.push_back({STM_OP_DIFF, j}); c.level.push_back(c.f + 1); }
-    for (int j = c.f + 1; j < l; ++j)
-      if (sig[l][j] != 0) {
-        c.ops.push_back({sig[l][j] == 1 ? STM_OP_AND : STM_OP_DIFF, j});
-        c.level.push_back(j + 1);
+    // codes in scan order: position j, then its out- / in-row (directed)
+    std::vector<int> codes;
+    for (int j = 0; j < l; ++j) {
+      codes.push_back(j);
+      if (directed) codes.push_back(j + 8);
+    }
+    size_t fi = 0;
+    while (fi < codes.size() && sig[l][codes[fi]] != 1) ++fi;
+    c.f = codes[fi];  // (the order is connected: some earlier position is adjacent)
+    for (size_t t = 0; t < fi; ++t)
+      if (sig[l][codes[t]] == -1) { c.ops.push_back({STM_OP_DIFF, codes[t]}); c.level.push_back((c.f & 7) + 1); }
+    for (size_t t = fi + 1; t < codes.size(); ++t)
+      if (sig[l][codes[t]] != 0) {
+        c.ops.push_back({sig[l][codes[t]] == 1 ? STM_OP_AND : STM_OP_DIFF, codes[t]});
+        c.level.push_back((codes[t] & 7) + 1);
       }
     if (!cm)
       for (auto& x : c.level) x = l;
@@ -337,7 +364,7 @@ extern "C" stm_status stm_pattern_compile(int k, int n_edges, const int32_t* edg
     int lazy_level = 0;  // lazy mode: once a chain op is unbounded for this consumer, it and the
                          // rest of the chain are computed at the consumer's level
     for (size_t t = 0; t < c.ops.size(); ++t) {
-      key.push_back(c.ops[t].first * 16 + c.ops[t].second);
+      key.push_back(c.ops[t].first * 16 + c.ops[t].second);  // (codes < 16)
       int level = c.level[t];
       if (lazy) {
         const unsigned known = (1u << c.level[t]) - 1;

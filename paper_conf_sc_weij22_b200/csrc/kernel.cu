@@ -366,12 +366,14 @@ __device__ __forceinline__ bool member(const int* __restrict__ a, int n, int x) 
 // neighbour > v, -1 = unknown), w = hub bitmap slot (-1 = none) -- one 16-byte load
 // instead of row_ptr[v], row_ptr[v+1], out_start[v] and hub_slot[v] from four arrays.
 __device__ __forceinline__ int4 vrec(const W& w, int v) { return __ldg(w.kp->vrec + v); }
-__device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len) {
-  const int4 r = vrec(w, v);
+// raw neighbour lists by position code (plan.h): dir 1 = the in-row of a directed graph
+// (its records follow the n out-row records, StmKParams::n_dir)
+__device__ __forceinline__ void row(const W& w, int v, const int*& p, int& len, int dir = 0) {
+  const int4 r = vrec(w, v + (dir ? w.kp->n_dir : 0));
   p = w.kp->col_idx + (unsigned)r.x;
   len = r.y;
 }
-__device__ __forceinline__ int degree(const W& w, int v) { return vrec(w, v).y; }
+__device__ __forceinline__ int degree(const W& w, int v, int dir = 0) { return vrec(w, v + (dir ? w.kp->n_dir : 0)).y; }
 
 // ----------------------------------------------------------------------------
 // plan access.  Single-pattern builds read the StmPlan; the STM_MULTI build reads the
@@ -440,7 +442,7 @@ __device__ __forceinline__ void node_slice(const W& w, int s, int F, int u, int 
 
 __device__ __forceinline__ void src_slice(const W& w, StmSrc src, int F, int u, int c, int un,
                                           const int*& p, int& len) {
-  if (src.kind == STM_SRC_RAW) row(w, pval(w, src.idx, F, u, c), p, len);
+  if (src.kind == STM_SRC_RAW) row(w, pval(w, src.idx & 7, F, u, c), p, len, src.idx >> 3);
   else node_slice(w, src.idx, F, u, un, p, len);
 }
 
@@ -500,8 +502,9 @@ __device__ __forceinline__ void narrow_split(int v, int s, const int*& p, int& n
 }
 
 // N(v) from its packed record, narrowed to (lo, hi); hub receives v's bitmap slot
-__device__ __forceinline__ void row_narrow(const W& w, int v, const int*& p, int& n, int& hub, int lo, int hi) {
-  const int4 r = vrec(w, v);
+__device__ __forceinline__ void row_narrow(const W& w, int v, const int*& p, int& n, int& hub, int lo, int hi,
+                                           int dir = 0) {
+  const int4 r = vrec(w, v + (dir ? w.kp->n_dir : 0));
   p = w.kp->col_idx + (unsigned)r.x;
   n = r.y;
   hub = r.w;
@@ -820,9 +823,9 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   J.op = cop;
   bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
   J.abm = -1;
-  if (ca.kind == STM_SRC_RAW) row_narrow(w, pval(w, ca.idx, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+  if (ca.kind == STM_SRC_RAW) row_narrow(w, pval(w, ca.idx & 7, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi, ca.idx >> 3);
   J.bbm = -1;
-  if (cop != STM_OP_NONE) row_narrow(w, pval(w, cb, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+  if (cop != STM_OP_NONE) row_narrow(w, pval(w, cb & 7, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi, cb >> 3);
   J.lab = f.lab;
   J.out = nullptr;
   J.u = u;
@@ -843,9 +846,10 @@ __device__ __forceinline__ Job count_job(const W& w, int F, int u, int c, int un
   bounds(w, f.lo, f.hi, F, u, c, J.lo, J.hi);
   J.abm = -1;
   if (P.cnt_a.kind == STM_SRC_RAW)
-    row_narrow(w, pval(w, P.cnt_a.idx, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+    row_narrow(w, pval(w, P.cnt_a.idx & 7, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi, P.cnt_a.idx >> 3);
   J.bbm = -1;
-  if (P.cnt_op != STM_OP_NONE) row_narrow(w, pval(w, P.cnt_b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+  if (P.cnt_op != STM_OP_NONE)
+    row_narrow(w, pval(w, P.cnt_b & 7, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi, P.cnt_b >> 3);
   J.lab = f.lab;
   J.out = nullptr;
   J.u = u;
@@ -938,8 +942,8 @@ __device__ int node_ub(const W& w, int s, int F, int u, int c) {
   int m = INT_MAX;
   for (;;) {
     const StmNode nd = pnode(w, s);
-    if (nd.op == STM_OP_AND) m = min(m, degree(w, pval(w, nd.b, F, u, c)));
-    if (nd.a_kind == STM_SRC_RAW) return min(m, degree(w, pval(w, nd.a, F, u, c)));
+    if (nd.op == STM_OP_AND) m = min(m, degree(w, pval(w, nd.b & 7, F, u, c), nd.b >> 3));
+    if (nd.a_kind == STM_SRC_RAW) return min(m, degree(w, pval(w, nd.a & 7, F, u, c), nd.a >> 3));
     if (pnode(w, nd.a).level == F + 1) { s = nd.a; continue; }
     const int* p;
     int len;
@@ -954,8 +958,9 @@ __device__ int node_ub_const(const W& w, int s, int F, int u) {
   int m = INT_MAX;
   for (;;) {
     const StmNode nd = pnode(w, s);
-    if (nd.op == STM_OP_AND && nd.b != F) m = min(m, degree(w, pval(w, nd.b, F, u, 0)));
-    if (nd.a_kind == STM_SRC_RAW) return nd.a != F ? min(m, degree(w, pval(w, nd.a, F, u, 0))) : m;
+    if (nd.op == STM_OP_AND && (nd.b & 7) != F) m = min(m, degree(w, pval(w, nd.b & 7, F, u, 0), nd.b >> 3));
+    if (nd.a_kind == STM_SRC_RAW)
+      return (nd.a & 7) != F ? min(m, degree(w, pval(w, nd.a & 7, F, u, 0), nd.a >> 3)) : m;
     if (pnode(w, nd.a).level == F + 1) { s = nd.a; continue; }
     const int* p;
     int len;
@@ -1043,10 +1048,11 @@ __device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {
         J.c = c;
         if (st < 0) bounds(w, cf.lo, cf.hi, F, u, c, J.lo, J.hi);  // the consumer's bounds
         else bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
-        if (nd.a_kind == STM_SRC_RAW) row_narrow(w, pval(w, nd.a, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+        if (nd.a_kind == STM_SRC_RAW)
+          row_narrow(w, pval(w, nd.a & 7, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi, nd.a >> 3);
         else node_slice(w, nd.a, F, u, t, J.A, J.alen);
         J.a_node = nd.a_kind == STM_SRC_NODE ? 1 : 0;
-        row_narrow(w, pval(w, nd.b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+        row_narrow(w, pval(w, nd.b & 7, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi, nd.b >> 3);
         J.op = nd.op;
         J.lab = st < 0 ? cf.lab : nd.lab;
         J.out = st < 0 ? nullptr : w.arena + (size_t)r * w.kp->cap + NOFF(w, r, t);
@@ -1123,10 +1129,11 @@ __device__ STEP_INL int build_nodes(W& w, int F, int m, bool prune) {  // single
         J.c = c;
         if (st < 0) bounds(w, cf.lo, cf.hi, F, u, c, J.lo, J.hi);  // the consumer's bounds
         else bounds(w, nd.lo, nd.hi, F, u, c, J.lo, J.hi);
-        if (nd.a_kind == STM_SRC_RAW) row_narrow(w, pval(w, nd.a, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi);
+        if (nd.a_kind == STM_SRC_RAW)
+          row_narrow(w, pval(w, nd.a & 7, F, u, c), J.A, J.alen, J.abm, J.lo, J.hi, nd.a >> 3);
         else node_slice(w, nd.a, F, u, t, J.A, J.alen);
         J.a_node = nd.a_kind == STM_SRC_NODE ? P.nodes[nd.a].level + 1 : 0;
-        row_narrow(w, pval(w, nd.b, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi);
+        row_narrow(w, pval(w, nd.b & 7, F, u, c), J.B, J.blen, J.bbm, J.lo, J.hi, nd.b >> 3);
         J.op = nd.op;
         J.lab = st < 0 ? cf.lab : nd.lab;
         J.out = st < 0 ? nullptr : w.arena + (size_t)s * w.kp->cap + NOFF(w, s, t);
@@ -1730,7 +1737,7 @@ __device__ __noinline__ void adopt_task(const StmKParams& kp, const StmTask& T) 
 #endif
     }
     __syncwarp();
-    if (i >= 2) {
+    if (i >= 2 || !STM_MULTI) {  // (i = 1: level-1 set nodes of directed plans, if any)
       int nb, ne, nst;
       bset(w, i - 1, w.h->cur[i - 1], nb, ne, nst);
       HDR_SYNC();  // every lane has read the header fields lane 0 rewrites
@@ -2132,6 +2139,18 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
           w.h->cur[1] = 0;
         }
         __syncwarp();
+#if !STM_MULTI
+        if (P.level_begin[1] != P.level_begin[2]) {
+          // level-1 set nodes (directed plans: e.g. N+(v0) & N-(v0) for a mutual arc), built
+          // per root (root_batch is 1 for such plans: offset 0 in every node region)
+          HDR_SYNC();
+          if (w.lane == 0)
+            for (int s = P.level_begin[1]; s < P.level_begin[2]; ++s) NOFF(w, s, 0) = 0;
+          __syncwarp();
+          m = build_nodes(w, 0, m, true);
+          if (m == 0) continue;  // the root cannot be extended: next root
+        }
+#endif
         PROF_BEGIN(1)
         set_sibling(w, 1, 0);
         PROF_END(1, 1)

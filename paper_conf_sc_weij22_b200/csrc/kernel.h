@@ -110,6 +110,7 @@ struct StmKParams {
   // handed out as several independent pieces from the start.  NULL: root space = vertex ids.
   const int2* entries;
   int32_t root_split;
+  int32_t n_dir;                  // directed graphs: vertex v's in-row is record v + n_dir (= n); 0 otherwise
   // Work-balanced chunks (stm_tuning.chunk_cost): chunk c is root-space positions
   // [chunk_bounds[c], chunk_bounds[c + 1]); NULL: fixed chunks of `chunk` positions.
   const int32_t* chunk_bounds;

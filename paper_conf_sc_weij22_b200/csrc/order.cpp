@@ -105,6 +105,8 @@ bool eval(const Model& m, const int* pi, double* cost, double* est) {
 stm_status build_model(int k, int n_edges, const int32_t* edges, const int32_t* labels, int n_restr,
                        const int32_t* restr, uint32_t flags, const stm_graph_stats* s, Model* m,
                        std::vector<int>* greedy) {
+  if (flags & STM_DIRECTED)
+    return stm_fail(STM_EUNSUPPORTED, "cost-based orders model undirected patterns only (directed: greedy order)");
   if (!s) return stm_fail(STM_EINVAL, "stats is NULL");
   if (s->n < 0 || s->nnz < 0) return stm_fail(STM_EINVAL, "stats: negative n or nnz");
   if (s->n_labels < 0 || s->n_labels > STM_STATS_LABELS) return stm_fail(STM_EINVAL, "stats: bad n_labels");

@@ -38,12 +38,12 @@ struct StmNode {
   int8_t level;     // computed when entering this level
   int8_t stage;     // dependency stage within the level (0 = operands from earlier levels)
   int8_t a_kind;    // STM_SRC_NODE / STM_SRC_RAW
-  int8_t b;         // level position of N(v_b)
+  int8_t b;         // position code of N(v_b): j (+ 8 for the in-row of a directed plan)
   int8_t op;        // STM_OP_AND / STM_OP_DIFF
   uint8_t lab;      // label-slot mask (STM_LAB_ANY = no label filter)
   uint8_t lo;       // bitmask of positions j: keep w > v_j
   uint8_t hi;       // bitmask of positions j: keep w < v_j
-  int16_t a;        // node index (merged plans: pool index) or level position of N(v_a)
+  int16_t a;        // node index (merged plans: pool index) or position code of N(v_a)
   uint8_t pad[2];
 };
 
@@ -56,7 +56,7 @@ struct StmFilter {
 struct StmSrc {
   int8_t kind;  // STM_SRC_NODE / STM_SRC_RAW
   int8_t pad;
-  int16_t idx;  // node index (merged plans: pool index) or level position
+  int16_t idx;  // node index (merged plans: pool index) or position code (j, + 8: in-row)
 };
 
 struct StmPlan {
@@ -74,9 +74,10 @@ struct StmPlan {
   StmFilter filt[STM_KMAX];          // candidate filter of levels 0..k-1
   // final (count) operation at level k-1: count |A op N(v_b)| under filt[k-1]
   StmSrc cnt_a;
-  int8_t cnt_b;                      // position, or -1 when op == STM_OP_NONE
+  int8_t cnt_b;                      // position code, or -1 when op == STM_OP_NONE
   int8_t cnt_op;
-  int8_t pad[2];
+  int8_t directed;                   // 1: raw operands name out- (code j) or in-rows (code j + 8)
+  int8_t pad;
   // Candidate-set pruning: need[l] = the minimal size of level l's
   // candidate set (within its bounds) for any embedding to extend the prefix -- v_l itself
   // plus every later v_m that must also come from it; a sibling whose level-(l) set is

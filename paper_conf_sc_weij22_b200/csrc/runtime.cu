@@ -72,6 +72,11 @@ struct DeviceGuard {
 struct stm_graph {
   int device = 0;
   int64_t n = 0, nnz = 0, max_degree = 0;
+  // Directed graphs (stm_graph_load_directed; NEXT-4): the CSR holds 2n rows, vertex v's
+  // out-row at row v and its in-row at row n + v (kernel StmKParams::n_dir).  No degree-
+  // ranked copy, hub bitmaps or root splitting for them (speed-only features).
+  bool directed = false;
+  int64_t n_rows = 0;
   int64_t* d_row_ptr = nullptr;
   int32_t* d_col_idx = nullptr;
   uint8_t* d_labels = nullptr;
@@ -234,25 +239,28 @@ static void query_persist(stm_graph* g) {
 }
 
 // ---------------------------------------------------------------- out_start
-__global__ void out_start_fill(const int64_t* rp, const int32_t* ci, int64_t n, int32_t* out) {
+// per row: index of the first entry > the row's vertex (row r is vertex r, or r - nv for
+// the in-rows of a directed graph)
+__global__ void out_start_fill(const int64_t* rp, const int32_t* ci, int64_t n, int64_t nv, int32_t* out) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t x = v < nv ? v : v - nv;
     int64_t lo = rp[v], hi = rp[v + 1];
     const int64_t b = lo;
     while (lo < hi) {
       const int64_t mid = (lo + hi) >> 1;
-      if (ci[mid] <= v) lo = mid + 1; else hi = mid;
+      if (ci[mid] <= x) lo = mid + 1; else hi = mid;
     }
     out[v] = (int32_t)(lo - b);
   }
 }
 
-static int32_t* build_out_start(const int64_t* rp, const int32_t* ci, int64_t n) {
+static int32_t* build_out_start(const int64_t* rp, const int32_t* ci, int64_t n, int64_t nv) {
   int32_t* d = nullptr;
   if (n < 1 || cudaMalloc(&d, sizeof(int32_t) * n) != cudaSuccess) {
     cudaGetLastError();
     return nullptr;
   }
-  out_start_fill<<<(unsigned)std::min<int64_t>((n + 255) / 256, 8192), 256>>>(rp, ci, n, d);
+  out_start_fill<<<(unsigned)std::min<int64_t>((n + 255) / 256, 8192), 256>>>(rp, ci, n, nv, d);
   if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
     cudaGetLastError();
     cudaFree(d);
@@ -490,9 +498,12 @@ static const stm_graph::HubBitmaps* ensure_hub(stm_graph* g, bool ranked, int mi
       h.n_hubs = h.words = 0;
     }
   }
-  e = cudaMalloc(&h.vrec, sizeof(int4) * (size_t)std::max<int64_t>(n, 1));
-  if (e == cudaSuccess && n > 0) {
-    vrec_fill<<<grid, 256>>>(rp, n, ranked ? g->d_rout_start : g->d_out_start, h.slot, h.vrec);
+  // one record per CSR row (directed graphs: out-rows then in-rows; no bitmaps there)
+  const int64_t nr = g->n_rows;
+  e = cudaMalloc(&h.vrec, sizeof(int4) * (size_t)std::max<int64_t>(nr, 1));
+  if (e == cudaSuccess && nr > 0) {
+    vrec_fill<<<(unsigned)std::min<int64_t>((nr + 255) / 256, 4096), 256>>>(
+        rp, nr, ranked ? g->d_rout_start : g->d_out_start, g->directed ? nullptr : h.slot, h.vrec);
     e = cudaGetLastError();
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
   }
@@ -505,7 +516,7 @@ static const stm_graph::HubBitmaps* ensure_hub(stm_graph* g, bool ranked, int mi
   return &h;
 }
 
-static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci) {
+static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci, bool symmetric) {
   if (rp[0] != 0) return stm_fail(STM_EINVAL, "row_ptr[0] != 0");
   for (int64_t v = 0; v < n; ++v)
     if (rp[v + 1] < rp[v]) return stm_fail(STM_EINVAL, "row_ptr decreases at %lld", (long long)v);
@@ -522,6 +533,7 @@ static stm_status validate_csr(int64_t n, const int64_t* rp, const int32_t* ci) 
           if (w < 0 || w >= n) { bad[t] = 1; badv[t] = v; break; }
           if (w == v) { bad[t] = 2; badv[t] = v; break; }
           if (e > rp[v] && ci[e - 1] >= w) { bad[t] = 3; badv[t] = v; break; }
+          if (!symmetric) continue;
           // symmetry: v must be in N(w)
           const int32_t* b = ci + rp[w];
           const int32_t* x = std::lower_bound(b, ci + rp[w + 1], (int32_t)v);
@@ -551,25 +563,19 @@ static stm_status dense_labels(int64_t n, const int32_t* labels, std::vector<uin
   return STM_OK;
 }
 
-extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
-                                     const int32_t* labels, int device, stm_graph** out) {
-  if (!out) return stm_fail(STM_EINVAL, "out is NULL");
-  if (n < 0 || n > INT32_MAX - 1) return stm_fail(STM_EINVAL, "n=%lld out of range", (long long)n);
-  if (!row_ptr) return stm_fail(STM_EINVAL, "row_ptr is NULL");
-  int64_t nnz = row_ptr[n];
-  if (nnz > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
-  if (nnz > (int64_t)UINT32_MAX)  // packed vertex records hold 32-bit row starts (kernel.cu vrec)
-    return stm_fail(STM_EUNSUPPORTED, "%lld adjacency entries >= 2^32", (long long)nnz);
-  stm_status s = validate_csr(n, row_ptr, col_idx);
-  if (s != STM_OK) return s;
+// Upload a validated CSR of n_rows rows over n vertices (n_rows = 2n for a directed graph:
+// out-rows then in-rows) and build the per-graph structures.
+static stm_status upload_graph(int64_t n, int64_t n_rows, const int64_t* row_ptr, const int32_t* col_idx,
+                               const int32_t* labels, int device, bool directed, stm_graph** out) {
+  const int64_t nnz = row_ptr[n_rows];
   std::vector<uint8_t> dense;
   std::vector<int32_t> values;
   if (labels) {
-    s = dense_labels(n, labels, dense, values);
+    stm_status s = dense_labels(n, labels, dense, values);
     if (s != STM_OK) return s;
   }
   int64_t maxd = 0;
-  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, row_ptr[v + 1] - row_ptr[v]);
+  for (int64_t v = 0; v < n_rows; ++v) maxd = std::max(maxd, row_ptr[v + 1] - row_ptr[v]);
   int ndev = 0;
   CU(cudaGetDeviceCount(&ndev));
   if (device < 0 || device >= ndev) return stm_fail(STM_EINVAL, "device %d of %d", device, ndev);
@@ -578,13 +584,15 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
   if (!g) return stm_fail(STM_ENOMEM, "host allocation");
   g->device = device;
   g->n = n;
+  g->n_rows = n_rows;
+  g->directed = directed;
   g->nnz = nnz;
   g->max_degree = maxd;
   g->label_values = values;
-  cudaError_t e = cudaMalloc(&g->d_row_ptr, sizeof(int64_t) * (n + 1));
+  cudaError_t e = cudaMalloc(&g->d_row_ptr, sizeof(int64_t) * (n_rows + 1));
   if (e == cudaSuccess) e = cudaMalloc(&g->d_col_idx, sizeof(int32_t) * std::max<int64_t>(nnz, 1));
   if (e == cudaSuccess && labels) e = cudaMalloc(&g->d_labels, std::max<int64_t>(n, 1));
-  if (e == cudaSuccess) e = cudaMemcpy(g->d_row_ptr, row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(g->d_row_ptr, row_ptr, sizeof(int64_t) * (n_rows + 1), cudaMemcpyHostToDevice);
   if (e == cudaSuccess && nnz) e = cudaMemcpy(g->d_col_idx, col_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice);
   if (e == cudaSuccess && labels && n) e = cudaMemcpy(g->d_labels, dense.data(), n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
@@ -595,12 +603,52 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
                     cudaGetErrorString(e));
   }
-  g->has_stats = stm_graph_stats_host(n, row_ptr, labels, &g->stats) == STM_OK;
-  build_ranked(g);
-  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
-  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
+  if (!directed) {
+    g->has_stats = stm_graph_stats_host(n, row_ptr, labels, &g->stats) == STM_OK;
+    build_ranked(g);
+  }
+  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n_rows, g->n);
+  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n, g->n);
   *out = g;
   return STM_OK;
+}
+
+extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                                     const int32_t* labels, int device, stm_graph** out) {
+  if (!out) return stm_fail(STM_EINVAL, "out is NULL");
+  if (n < 0 || n > INT32_MAX - 1) return stm_fail(STM_EINVAL, "n=%lld out of range", (long long)n);
+  if (!row_ptr) return stm_fail(STM_EINVAL, "row_ptr is NULL");
+  int64_t nnz = row_ptr[n];
+  if (nnz > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
+  if (nnz > (int64_t)UINT32_MAX)  // packed vertex records hold 32-bit row starts (kernel.cu vrec)
+    return stm_fail(STM_EUNSUPPORTED, "%lld adjacency entries >= 2^32", (long long)nnz);
+  stm_status s = validate_csr(n, row_ptr, col_idx, true);
+  if (s != STM_OK) return s;
+  return upload_graph(n, n, row_ptr, col_idx, labels, device, false, out);
+}
+
+extern "C" stm_status stm_graph_load_directed(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                                              const int32_t* labels, int device, stm_graph** out) {
+  if (!out) return stm_fail(STM_EINVAL, "out is NULL");
+  if (n < 0 || n > INT32_MAX - 1) return stm_fail(STM_EINVAL, "n=%lld out of range", (long long)n);
+  if (!row_ptr) return stm_fail(STM_EINVAL, "row_ptr is NULL");
+  const int64_t m = row_ptr[n];
+  if (m > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
+  if (2 * m > (int64_t)UINT32_MAX) return stm_fail(STM_EUNSUPPORTED, "%lld arcs: 2m >= 2^32", (long long)m);
+  stm_status s = validate_csr(n, row_ptr, col_idx, false);
+  if (s != STM_OK) return s;
+  // rows 0..n-1: the out-rows as given; rows n..2n-1: the in-rows (transpose, sorted)
+  std::vector<int64_t> rp(2 * n + 1, 0);
+  std::vector<int32_t> ci(2 * m);
+  for (int64_t v = 0; v <= n; ++v) rp[v] = row_ptr[v];
+  std::vector<int64_t> indeg(n + 1, 0);
+  for (int64_t e = 0; e < m; ++e) ++indeg[col_idx[e]];
+  for (int64_t v = 0; v < n; ++v) rp[n + v + 1] = rp[n + v] + indeg[v];
+  std::copy(col_idx, col_idx + m, ci.begin());
+  std::vector<int64_t> fill(rp.begin() + n, rp.begin() + 2 * n);
+  for (int64_t v = 0; v < n; ++v)  // sources in increasing order: each in-row comes out sorted
+    for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) ci[fill[col_idx[e]]++] = (int32_t)v;
+  return upload_graph(n, 2 * n, rp.data(), ci.data(), labels, device, true, out);
 }
 
 extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_t* d_row_ptr,
@@ -639,6 +687,7 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
   if (!g) return stm_fail(STM_ENOMEM, "host allocation");
   g->device = device;
   g->n = n;
+  g->n_rows = n;
   g->nnz = nnz;
   g->max_degree = maxd;
   g->owns_csr = false;
@@ -671,8 +720,8 @@ extern "C" stm_status stm_graph_load_device(int64_t n, int64_t nnz, const int64_
     cudaGetLastError();
   }
   build_ranked(g);
-  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n);
-  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n);
+  g->d_out_start = build_out_start(g->d_row_ptr, g->d_col_idx, g->n_rows, g->n);
+  if (g->ranked) g->d_rout_start = build_out_start(g->d_rrow_ptr, g->d_rcol_idx, g->n, g->n);
   *out = g;
   return STM_OK;
 }
@@ -773,6 +822,9 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.jit < -1 || t.jit > 1) return stm_fail(STM_EINVAL, "jit %d not in -1..1", t.jit);
   if (d_result && ((uintptr_t)d_result & 7)) return stm_fail(STM_EINVAL, "d_result not 8-byte aligned");
   const StmPlan& P = p->dev;
+  if ((P.directed != 0) != g->directed)
+    return stm_fail(STM_EINVAL, g->directed ? "directed graph needs a STM_DIRECTED plan"
+                                             : "STM_DIRECTED plan on an undirected graph");
   if (!p->labels.empty() && !g->d_labels) {
     bool any = false;
     for (int x : p->labels) any |= x >= 0;
@@ -795,6 +847,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   kp.root_map = use_rank ? g->d_rank2orig : nullptr;
   kp.split = t.narrow_split == 0 ? 1 : 0;
   kp.n = g->n;
+  kp.n_dir = g->directed ? (int32_t)g->n : 0;
   if (la) {
     kp.root_lo = la->root_lo;
     kp.n = la->root_hi;
@@ -814,7 +867,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
     // root splitting (stm_tuning.root_split): not for listing pages, which are root-id ranges
     const int T = t.root_split == 0 ? STM_ROOT_SPLIT_AUTO : t.root_split;
     const stm_graph::RootEntries* E = nullptr;
-    if (!la && T > 0) {
+    if (!la && T > 0 && !g->directed) {
       E = ensure_entries(g, use_rank, T);
       if (E) {
         kp.entries = E->d;
@@ -889,6 +942,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   glock.unlock();
   // roots gathered per frame-1 batch: with work-balanced chunks a light chunk holds many roots
   kp.root_batch = (kp.chunk_bounds && t.root_chunk == 0) ? STM_RMAX : std::max(1, std::min(STM_RMAX, root_chunk));
+  if (P.level_begin[1] != P.level_begin[2]) kp.root_batch = 1;  // level-1 set nodes: built per root (kernel.cu)
   kp.count_bytes = t.instrument ? 1 : 0;
   if (t.hash_slots < 0 || t.hash_slots > 4096 || (t.hash_slots && (t.hash_slots < 64 || (t.hash_slots & (t.hash_slots - 1)))))
     return stm_fail(STM_EINVAL, "hash_slots %d: 0 or a power of two in 64..4096", t.hash_slots);

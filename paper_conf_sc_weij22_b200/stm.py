@@ -18,6 +18,7 @@ STM_OK, STM_EINVAL, STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED, STM_EOVERFLOW, STM_
 STM_EDGE_INDUCED, STM_VERTEX_INDUCED, STM_NO_CODE_MOTION, STM_AUTO_RESTRICT, STM_AUTO_ORDER = 0, 1, 2, 4, 8
 STM_LAZY_UNBOUNDED = 16
 STM_CENSUS_PER_MOTIF = 32
+STM_DIRECTED = 64
 _NAMES = {1: "STM_EINVAL", 2: "STM_ENOMEM", 3: "STM_ECUDA", 4: "STM_EUNSUPPORTED", 5: "STM_EOVERFLOW",
           6: "STM_ETIMEOUT"}
 STM_IPC_HANDLE_BYTES = 64
@@ -29,7 +30,7 @@ EXPORTS = ["stm_match_list", "stm_graph_load", "stm_graph_load_device", "stm_gra
            "stm_graph_stats_host", "stm_order_cost", "stm_order_optimize", "stm_motif_catalog",
            "stm_motif_census", "stm_cursors_alloc", "stm_cursors_open", "stm_cursors_close", "stm_cursors_free",
            "stm_cursors_reset", "stm_graph_get_stats", "stm_motif_census_launches", "stm_motif_merge_stats",
-           "stm_plan_raw"]
+           "stm_plan_raw", "stm_graph_load_directed"]
 
 
 class StmError(RuntimeError):
@@ -90,6 +91,7 @@ def _load():
     P64 = ctypes.POINTER(ctypes.c_int64)
     sig = {
         "stm_graph_load": [i64, vp, vp, vp, i32, ctypes.POINTER(vp)],
+        "stm_graph_load_directed": [i64, vp, vp, vp, i32, ctypes.POINTER(vp)],
         "stm_graph_load_device": [i64, i64, vp, vp, vp, i32, ctypes.POINTER(vp)],
         "stm_graph_info": [vp, P64, P64, P64],
         "stm_graph_free": [vp],
@@ -154,6 +156,14 @@ def stm_graph_load(n: int, row_ptr, col_idx, labels=None, device: int = 0) -> in
     rp, ci, lb = _arr(row_ptr, np.int64), _arr(col_idx, np.int32), _arr(labels, np.int32)
     h = ctypes.c_void_p()
     _check(lib.stm_graph_load(n, _p(rp), _p(ci), _p(lb), device, ctypes.byref(h)))
+    return h.value
+
+
+def stm_graph_load_directed(n: int, row_ptr, col_idx, labels=None, device: int = 0) -> int:
+    """Directed graph from its out-neighbour rows (NEXT-4)."""
+    rp, ci, lb = _arr(row_ptr, np.int64), _arr(col_idx, np.int32), _arr(labels, np.int32)
+    h = ctypes.c_void_p()
+    _check(lib.stm_graph_load_directed(n, _p(rp), _p(ci), _p(lb), device, ctypes.byref(h)))
     return h.value
 
 
@@ -423,10 +433,12 @@ def stm_last_launch() -> dict:
 class Graph:
     """Device-resident data graph (owns the stm_graph handle)."""
 
-    def __init__(self, n: int, row_ptr, col_idx, labels=None, device: int = 0):
-        self.handle = stm_graph_load(n, row_ptr, col_idx, labels, device)
+    def __init__(self, n: int, row_ptr, col_idx, labels=None, device: int = 0, directed: bool = False):
+        """directed: row_ptr / col_idx are out-neighbour rows of a digraph (stm_graph_load_directed)."""
+        self.handle = (stm_graph_load_directed if directed else stm_graph_load)(n, row_ptr, col_idx, labels, device)
         self.n, self.nnz, self.max_degree = stm_graph_info(self.handle)
         self.device = device
+        self.directed = directed
 
     @classmethod
     def from_stmgen(cls, g, device: int = 0) -> "Graph":
@@ -449,18 +461,22 @@ class Plan:
 
     def __init__(self, k: int, edges, labels=None, order=None, restrictions=None, vertex_induced=False,
                  code_motion=True, auto_restrict=None, auto_order=False, lazy_unbounded=False,
-                 cost_stats: Optional[stm_graph_stats] = None, graph: Optional["Graph"] = None):
+                 cost_stats: Optional[stm_graph_stats] = None, graph: Optional["Graph"] = None,
+                 directed: bool = False):
         """cost_stats: graph statistics (stm_graph_stats_host) -> the cost-optimal order (NEXT-2)
         replaces `order`.  graph: compile for this loaded graph -- its statistics (stm_graph_get_stats)
-        give the cost-based order unless `order` or `cost_stats` is given."""
-        if graph is not None and cost_stats is None and order is None and not auto_order:
+        give the cost-based order unless `order` or `cost_stats` is given.  directed: `edges` are arcs
+        (a, b) = a -> b (STM_DIRECTED; graphs from Graph(..., directed=True)); greedy order only."""
+        directed = directed or bool(graph is not None and getattr(graph, "directed", False))
+        if graph is not None and cost_stats is None and order is None and not auto_order and not directed:
             cost_stats = stm_graph_get_stats(graph.handle)
         if auto_restrict is None:
             auto_restrict = restrictions is None
         flags = (STM_VERTEX_INDUCED if vertex_induced else 0) | (0 if code_motion else STM_NO_CODE_MOTION)
         flags |= STM_AUTO_RESTRICT if auto_restrict else 0
         flags |= STM_LAZY_UNBOUNDED if lazy_unbounded else 0
-        if cost_stats is not None:
+        flags |= STM_DIRECTED if directed else 0
+        if cost_stats is not None and not directed:
             order, self.model_cost, self.model_count = stm_order_optimize(k, edges, labels, restrictions, flags,
                                                                           cost_stats)
         flags |= STM_AUTO_ORDER if auto_order else 0

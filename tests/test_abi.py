@@ -190,3 +190,16 @@ def test_lazy_unbounded_plan_k6_minus_e(stm):
     # cliques are bounded at every level: lazy changes nothing
     k5 = CATALOG["k5"]
     assert _plan_lines(stm, k5.k, k5.edges, lazy_unbounded=True)[1][2:] == _plan_lines(stm, k5.k, k5.edges)[1][2:]
+
+
+def test_directed_plan_compile():
+    """STM_DIRECTED plans (NEXT-4): raw operands name out-rows N+(v) or in-rows N-(v); the directed
+    3-cycle counts N-(v0) & N+(v1) at its last level, with |Aut| = 3 (rotations only)."""
+    from paper_conf_sc_weij22_b200 import stm
+    p = stm.Plan(3, [(0, 1), (1, 2), (2, 0)], directed=True)
+    d = p.describe()
+    assert "directed" in d and p.aut == 3
+    assert "count 2: N-(v0) & N+(v1)" in d
+    assert stm.Plan(3, [(0, 1), (1, 2), (0, 2)], directed=True).aut == 1
+    # an undirected plan never carries in-rows
+    assert "N-(" not in stm.Plan(3, [(0, 1), (1, 2), (0, 2)]).describe()
