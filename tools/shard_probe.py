@@ -39,6 +39,13 @@ for name in pats:
                 best = min(best, time.perf_counter() - t0)
             times.append(best)
             cnt += c
+            if r == 0 and W > 1 and os.environ.get("STM_LIB_PATH", "").endswith("prof.so"):
+                prof = stm.stm_last_profile()
+                tl = prof["timeline_busy_warps"]
+                last = max([i for i, x in enumerate(tl) if x > 0] or [0])
+                print(f"   W={W} rank 0 busy warps per 0.5 ms: " + " ".join(f"{x:.0f}" for x in tl[:last + 1]), flush=True)
+                print(f"   tail: cursors dry at max {prof['tail']['max_dry'] / 1.9e6:.2f} ms, "
+                      f"indivisible {prof['max_task_cycles'] / 1.9e6:.2f} ms", flush=True)
         if total is None:
             total, t1 = cnt, max(times)
         ok = "ok" if cnt == total else f"MISMATCH {cnt} != {total}"
