@@ -139,6 +139,60 @@ __global__ void degree_scan(const int64_t* rp, int64_t n, long long* out) {
   }
 }
 
+// Full CSR validation on the device (stm_graph_load): one thread per adjacency entry checks
+// the id range, no self-loop, strict increase within the row and (symmetric graphs) that
+// the reverse entry exists (binary search in the neighbour's row).  bad[r] = the smallest
+// offending vertex for reason r (1 range, 2 self-loop, 3 order, 4 symmetry); INT64_MAX = none.
+__global__ void validate_entries(const int64_t* rp, const int32_t* ci, int64_t n, int symmetric,
+                                 unsigned long long* bad) {
+  const int64_t nnz = rp[n];
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
+    // the row of entry e: binary search in row_ptr
+    int64_t lo = 0, hi = n;
+    while (hi - lo > 1) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (rp[mid] <= e) lo = mid; else hi = mid;
+    }
+    const int64_t v = lo;
+    const int64_t w = ci[e];
+    int why = 0;
+    if (w < 0 || w >= n) why = 1;
+    else if (w == v) why = 2;
+    else if (e > rp[v] && ci[e - 1] >= w) why = 3;
+    else if (symmetric) {
+      int64_t a = rp[w], b = rp[w + 1];
+      while (a < b) {
+        const int64_t mid = (a + b) >> 1;
+        if (ci[mid] < v) a = mid + 1; else b = mid;
+      }
+      if (a == rp[w + 1] || ci[a] != v) why = 4;
+    }
+    if (why) atomicMin(&bad[why], (unsigned long long)v);
+  }
+}
+
+static stm_status validate_on_device(const int64_t* d_rp, const int32_t* d_ci, int64_t n, int64_t nnz,
+                                     bool symmetric) {
+  if (nnz == 0) return STM_OK;
+  unsigned long long* d = nullptr;
+  CU(cudaMalloc(&d, 5 * sizeof(unsigned long long)));
+  unsigned long long h[5];
+  for (auto& x : h) x = ~0ull;
+  cudaError_t e = cudaMemcpy(d, h, sizeof h, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) {
+    validate_entries<<<(unsigned)std::min<int64_t>((nnz + 255) / 256, 8192), 256>>>(d_rp, d_ci, n, symmetric ? 1 : 0, d);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaMemcpy(h, d, sizeof h, cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  if (e != cudaSuccess) return stm_fail(STM_ECUDA, "CSR validation: %s", cudaGetErrorString(e));
+  static const char* why[] = {"", "neighbour id out of range", "self-loop", "row not strictly increasing",
+                              "graph not symmetric"};
+  for (int r = 1; r < 5; ++r)
+    if (h[r] != ~0ull) return stm_fail(STM_EINVAL, "%s at vertex %lld", why[r], (long long)h[r]);
+  return STM_OK;
+}
+
 // ---------------------------------------------------------------- degree-ranked copy
 __global__ void rank_keys(const int64_t* rp, int64_t n, unsigned long long* keys) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
@@ -566,7 +620,8 @@ static stm_status dense_labels(int64_t n, const int32_t* labels, std::vector<uin
 // Upload a validated CSR of n_rows rows over n vertices (n_rows = 2n for a directed graph:
 // out-rows then in-rows) and build the per-graph structures.
 static stm_status upload_graph(int64_t n, int64_t n_rows, const int64_t* row_ptr, const int32_t* col_idx,
-                               const int32_t* labels, int device, bool directed, stm_graph** out) {
+                               const int32_t* labels, int device, bool directed, stm_graph** out,
+                               bool validate_symmetric = false) {
   const int64_t nnz = row_ptr[n_rows];
   std::vector<uint8_t> dense;
   std::vector<int32_t> values;
@@ -603,6 +658,13 @@ static stm_status upload_graph(int64_t n, int64_t n_rows, const int64_t* row_ptr
     return stm_fail(e == cudaErrorMemoryAllocation ? STM_ENOMEM : STM_ECUDA, "graph upload: %s",
                     cudaGetErrorString(e));
   }
+  if (validate_symmetric) {  // the entry checks of stm_graph_load, on the uploaded copy
+    const stm_status vs = validate_on_device(g->d_row_ptr, g->d_col_idx, n, nnz, true);
+    if (vs != STM_OK) {
+      stm_graph_free(g);
+      return vs;
+    }
+  }
   if (!directed) {
     g->has_stats = stm_graph_stats_host(n, row_ptr, labels, &g->stats) == STM_OK;
     build_ranked(g);
@@ -622,9 +684,12 @@ extern "C" stm_status stm_graph_load(int64_t n, const int64_t* row_ptr, const in
   if (nnz > 0 && !col_idx) return stm_fail(STM_EINVAL, "col_idx is NULL");
   if (nnz > (int64_t)UINT32_MAX)  // packed vertex records hold 32-bit row starts (kernel.cu vrec)
     return stm_fail(STM_EUNSUPPORTED, "%lld adjacency entries >= 2^32", (long long)nnz);
-  stm_status s = validate_csr(n, row_ptr, col_idx, true);
-  if (s != STM_OK) return s;
-  return upload_graph(n, n, row_ptr, col_idx, labels, device, false, out);
+  // row_ptr checks on the host (O(n)); the O(m log d) entry checks (range, self-loops, order,
+  // symmetry) on the device after the upload -- the same checks and messages as validate_csr
+  if (row_ptr[0] != 0) return stm_fail(STM_EINVAL, "row_ptr[0] != 0");
+  for (int64_t v = 0; v < n; ++v)
+    if (row_ptr[v + 1] < row_ptr[v]) return stm_fail(STM_EINVAL, "row_ptr decreases at %lld", (long long)v);
+  return upload_graph(n, n, row_ptr, col_idx, labels, device, false, out, true);
 }
 
 extern "C" stm_status stm_graph_load_directed(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,

@@ -121,3 +121,25 @@ def test_directed_mismatch_rejected(dg_hubs):
     d, G = dg_hubs
     with pytest.raises(stm.StmError):
         stm.count(G, stm.Plan(3, [(0, 1), (1, 2), (0, 2)]))  # undirected plan on a directed graph
+
+
+@pytest.mark.parametrize("rows,why", [
+    ([[1], []], "not symmetric"),                  # 0 -> 1 without 1 -> 0
+    ([[0, 1], [0]], "self-loop"),
+    ([[2, 1], [0], [0]], "strictly increasing"),
+    ([[1, 7], [0]], "out of range"),
+])
+def test_graph_validation(rows, why):
+    """stm_graph_load rejects what is not an undirected simple graph (entry checks on the device);
+    stm_graph_load_directed accepts one-way arcs but rejects the rest."""
+    n = len(rows)
+    rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int64)
+    ci = np.array([x for r in rows for x in r], dtype=np.int32)
+    with pytest.raises(stm.StmError) as ei:
+        stm.Graph(n, rp, ci)
+    assert ei.value.status == stm.STM_EINVAL and why in str(ei.value)
+    if why == "not symmetric":
+        stm.Graph(n, rp, ci, directed=True).close()
+    else:
+        with pytest.raises(stm.StmError):
+            stm.Graph(n, rp, ci, directed=True)
