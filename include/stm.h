@@ -87,8 +87,9 @@ enum { STM_K_MAX = 8 };
  *            At most 255 distinct values (STM_EUNSUPPORTED otherwise).
  *   device   CUDA device ordinal.
  *   out      receives the handle.
- * Errors: STM_EINVAL for any CSR violation above (the full check is O(m log d)
- * on the host), STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED (> 255 labels, or
+ * Errors: STM_EINVAL for any CSR violation above (row_ptr checked on the host, the
+ * O(m log d) entry checks on the device after the copy; no handle is returned on a
+ * violation), STM_ENOMEM, STM_ECUDA, STM_EUNSUPPORTED (> 255 labels, or
  * row_ptr[n] >= 2^32 adjacency entries: the kernel's packed per-vertex records hold
  * 32-bit row starts).
  */
