@@ -102,7 +102,8 @@
 #define STM_ELEM_NOINLINE 1 // 1: run_jobs' element loop is one out-of-line function (i-cache)
 #endif
 #ifndef STM_BM_CS
-#define STM_BM_CS 1         // 1: hub-bitmap probes as streaming loads (L2 evict-first; K6-e -3 %)
+#define STM_BM_CS 0         // 1: hub-bitmap probes as streaming loads (L2 evict-first): K6-e -3 % time
+                            //    but +17 % DRAM traffic (fewer L2 hits on re-probed words) -- off
 #endif
 #if STM_BM_CS
 #define STM_BM_LOAD(p) __ldcs(p)
