@@ -193,7 +193,8 @@ typedef struct stm_tuning {
                              in HBM, and set-operation probes into its list test one bit instead of
                              binary-searching.  0 = auto (64), -1 = off.  Built lazily on the first
                              launch that uses them and cached on the graph.  Speed only. */
-  int32_t bitmap_budget_mb;  /* at most this many MiB of bitmaps (highest degrees first); 0 = auto (2048). */
+  int32_t bitmap_budget_mb;  /* at most this many MiB of bitmaps (highest degrees first); 0 = auto (512:
+                             on C5 K6-e the same time as 2048 with half the DRAM traffic). */
   int32_t occupancy;      /* kernel register budget: 1 = 64 registers (32 warps/SM), 2 = 40 registers
                              (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
                              than half the L2.  Speed only.  Default 0. */

@@ -22,7 +22,7 @@
 
 // Hub bitmap defaults (stm_tuning 0 = auto): measured on B200, DESIGN.md "Hub bitmaps".
 #define STM_BITMAP_AUTO_MIN_DEGREE 64
-#define STM_BITMAP_AUTO_BUDGET_MB 2048
+#define STM_BITMAP_AUTO_BUDGET_MB 512   // (C5 K6-e: 2048 MB -> 512 MB same time, DRAM 54 -> 28 GB per launch)
 #define STM_L2_PERSIST_AUTO_MB 0   // measured neutral at 24-48 MiB, worse at 96 MiB on C5: off
 #define STM_CHUNK_COST_AUTO 512    // work-balanced root chunks (stm_tuning.chunk_cost)
 #define STM_ROOT_SPLIT_AUTO 512    // root splitting piece size (stm_tuning.root_split; measured 32..512 on C2-C5)
