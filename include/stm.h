@@ -177,7 +177,7 @@ typedef struct stm_tuning {
                              0 = auto (32 with the 40-register kernel, else 16; measured).  Default 0. */
   int32_t root_chunk;     /* roots per cursor grab, 1..32; 0 = auto (1 with the 64-register kernel,
                              2 with the 40-register one; measured on B200).  Default 0. */
-  int32_t block_warps;    /* warps per block, 1..32; 0 = default (16). */
+  int32_t block_warps;    /* warps per block, 1..32; 0 = default (32: larger blocks share work locally). */
   int32_t blocks_per_sm;  /* 0 = as many as fit (occupancy API). */
   int32_t instrument;     /* 1 = instrumented launch: count algorithmic bytes (stm_last_launch). Default 0. */
   int32_t hash_slots;     /* per-warp shared-memory hash set for operands shared by a combined set
@@ -195,8 +195,8 @@ typedef struct stm_tuning {
                              launch that uses them and cached on the graph.  Speed only. */
   int32_t bitmap_budget_mb;  /* at most this many MiB of bitmaps (highest degrees first); 0 = auto (512:
                              on C5 K6-e the same time as 2048 with half the DRAM traffic). */
-  int32_t occupancy;      /* kernel register budget: 1 = 64 registers (32 warps/SM), 2 = 40 registers
-                             (48 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
+  int32_t occupancy;      /* kernel register budget: 1 = 64 registers (32 warps/SM), 2 = 32 registers
+                             (64 warps/SM, more DRAM latency hidden); 0 = auto: 2 when the CSR is larger
                              than half the L2.  Speed only.  Default 0. */
   int32_t root_order;     /* order in which root chunks are handed out: 1 = ascending vertex id,
                              2 = descending (heavy roots first on the degree-ranked copy), 3 = work-

@@ -78,7 +78,7 @@
 #define GATHER_SLOW_INL __forceinline__
 #endif
 #ifndef STM_OCC_MAXT
-#define STM_OCC_MAXT 1536   // __launch_bounds__ of the high-occupancy variant (40 registers)
+#define STM_OCC_MAXT 2048   // __launch_bounds__ of the high-occupancy variant (32 registers, 64 warps/SM)
 #endif
 #ifndef STM_INSTR
 #define STM_INSTR 0         // 1: the instrumented build (kernel_instr.cu): algorithmic-byte / idle counters
@@ -2253,7 +2253,7 @@ __device__ __forceinline__ void stm_count_body(const StmKParams& kp) {
 }
 
 // Two register budgets of the same kernel (stm_tuning.occupancy): 64 registers ->
-// 32 resident warps per SM, or 40 registers (with spills) -> 48 warps per SM, which
+// 32 resident warps per SM, or 32 registers (with spills) -> 64 warps per SM, which
 // hides more DRAM latency when the graph does not fit in L2 (measured).
 #ifdef STM_NVRTC
 #define STM_KLINK extern "C"  // JIT builds: unmangled names for cudaLibraryGetKernel

@@ -156,7 +156,7 @@ int stm_hash_compiled();
 int stm_drive_compiled();
 // size in bytes of the dynamic shared memory for one block
 int stm_smem_bytes(int block_warps, int k, int n_nodes, int ht_slots);
-// kernel variants (register budgets): 1 = 64 registers, 2 = 40 registers (more warps)
+// kernel variants (register budgets): 1 = 64 registers, 2 = 32 registers (more warps)
 // launches the persistent kernel (cooperative); returns cudaError_t as int
 int stm_launch(int variant, const StmKParams& kp, int grid, void* stream);
 int stm_launch_instr(int variant, const StmKParams& kp, int grid, void* stream);  // instrumented build

@@ -844,7 +844,7 @@ extern "C" void stm_tuning_default(stm_tuning* t) {
   t->l2_persist_mb = 0;  // auto
   t->drive_ratio = 0;    // off (measured)
   t->root_chunk = 0;  // auto: 1 with the 64-register kernel, 2 with the 40-register one (measured)
-  t->block_warps = 16;
+  t->block_warps = 32;  // (measured: C2 K4 -11 %, C3 K5 -5 %, C5 K5 -6 %, K6-e -4 % vs 16)
   t->blocks_per_sm = 0;
   t->bitmap_min_degree = 0;  // auto
   t->bitmap_budget_mb = 0;   // auto
@@ -876,7 +876,7 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   if (t.occupancy < 0 || t.occupancy > 2) return stm_fail(STM_EINVAL, "occupancy %d not in 0..2", t.occupancy);
   if (t.root_order < 0 || t.root_order > 3) return stm_fail(STM_EINVAL, "root_order %d not in 0..3", t.root_order);
   if (t.root_chunk < 0) return stm_fail(STM_EINVAL, "root_chunk %d < 0", t.root_chunk);
-  if (t.block_warps == 0) t.block_warps = 16;
+  if (t.block_warps == 0) t.block_warps = 32;
   if (t.block_warps < 1 || t.block_warps > 32) return stm_fail(STM_EINVAL, "block_warps %d", t.block_warps);
   if (t.stop_level < 1) t.stop_level = 1;
   if (t.watchdog_ms < 0) return stm_fail(STM_EINVAL, "watchdog_ms %d < 0", t.watchdog_ms);
