@@ -19,6 +19,10 @@
  *   - Handles (stm_graph*, stm_plan*) are owned by the library and released by
  *     the matching *_free call.  Graphs and plans are immutable after creation
  *     and may be shared by concurrent calls on different CUDA streams.
+ *   - Per-launch scratch (set arena, scheduler state) is library-owned, cached per
+ *     (device, stream) for the life of the process and reused by every graph counted
+ *     on that stream; calls on ONE stream must therefore be issued from one host
+ *     thread at a time (their launches are stream-ordered).
  *   - CUDA failures map to STM_ECUDA (message carries cudaGetErrorString).
  *   - A count is never silently wrong: capacity problems are STM_EOVERFLOW.
  *

@@ -111,7 +111,6 @@ struct stm_graph {
   };
   std::map<std::tuple<int, int, int64_t>, HubBitmaps> hubs;  // (ranked, min_deg, budget) -> set
   std::mutex mu;
-  std::map<void*, Scratch> scratch;  // per stream
   // root entries per (numbering, piece size) (kernel.h StmKParams::entries), built lazily
   struct RootEntries {
     int2* d = nullptr;
@@ -809,10 +808,6 @@ extern "C" stm_status stm_graph_get_stats(const stm_graph* g, stm_graph_stats* o
 extern "C" stm_status stm_graph_free(stm_graph* g) {
   if (!g) return STM_OK;
   DeviceGuard dg(g->device);
-  for (auto& kv : g->scratch) {
-    cudaFree(kv.second.arena);
-    cudaFree(kv.second.state);
-  }
   if (g->owns_csr) {
     cudaFree(g->d_row_ptr);
     cudaFree(g->d_col_idx);
@@ -1048,10 +1043,15 @@ static stm_status launch(const stm_graph* gc, const stm_plan* p, const stm_tunin
   while ((1 << pool_shift) < 2 * grid) ++pool_shift;
   const size_t state_bytes = sizeof(StmWork) + 64 + sizeof(StmPoolSlot) * ((size_t)1 << pool_shift);
 
+  // per-launch scratch (set arena + scheduler state), cached per (device, stream) for the
+  // process and shared by every graph counted on that stream (stream order serialises its
+  // users): a new graph does not pay a multi-GB allocation on its first launch
   Scratch* S;
   {
-    std::lock_guard<std::mutex> lk(g->mu);
-    S = &g->scratch[stream];
+    static std::mutex scratch_mu;
+    static std::map<std::pair<int, void*>, Scratch> scratch_cache;
+    std::lock_guard<std::mutex> lk(scratch_mu);
+    S = &scratch_cache[std::make_pair(g->device, stream)];
     if (S->arena_bytes < arena_bytes) {
       cudaFree(S->arena);
       S->arena = nullptr;
