@@ -4,7 +4,9 @@ import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import stmgen
 from paper_conf_sc_weij22_b200 import stm
-for spec in sys.argv[1:]:
+tk = dict(a.split("=") for a in sys.argv[1:] if "=" in a)
+tuning = stm.stm_tuning_default(**{k: int(v) for k, v in tk.items()}) if tk else None
+for spec in [a for a in sys.argv[1:] if "=" not in a]:
     cfg, k = spec.split(":")[:2]
     k = int(k)
     flags = (stm.STM_VERTEX_INDUCED if ":vi" in spec else 0) | (stm.STM_AUTO_ORDER if ":greedy" in spec else 0)
@@ -12,11 +14,11 @@ for spec in sys.argv[1:]:
     G = stm.Graph.from_stmgen(g)
     res = {}
     for name, f in (("merged", flags), ("per-motif", flags | stm.STM_CENSUS_PER_MOTIF)):
-        stm.stm_motif_census(G.handle, k, f)  # warm-up
+        stm.stm_motif_census(G.handle, k, f, tuning=tuning)  # warm-up
         best = 1e9
         for _ in range(3):
             t0 = time.perf_counter()
-            c = stm.stm_motif_census(G.handle, k, f)
+            c = stm.stm_motif_census(G.handle, k, f, tuning=tuning)
             best = min(best, time.perf_counter() - t0)
         res[name] = c
         print(f"{spec:10} {name:9} {len(c)} motifs in {stm.stm_motif_census_launches()} launch(es) "
