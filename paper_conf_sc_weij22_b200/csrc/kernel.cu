@@ -113,6 +113,9 @@
 #ifndef STM_BATCH_ELEMS
 #define STM_BATCH_ELEMS 0   // > 0: admit siblings into a batch only while the summed set-size
 #endif                      //    bounds stay within this many elements (0: the arena region)
+#ifndef STM_DEEP_FRAC
+#define STM_DEEP_FRAC 8     // every frame is donated while more than 1/STM_DEEP_FRAC of the warps idle
+#endif
 #ifndef STM_GCHK_CYCLES
 #define STM_GCHK_CYCLES 4096  // busy warps look at the pool's demand at most this often (SM cycles)
 #endif
@@ -879,7 +882,7 @@ __device__ __forceinline__ bool pool_wanted(const W& w) {
       w.h->gchk = now;
       volatile StmWork* vw = w.kp->work;
       want = vw->deficit > 0;
-      w.h->deep = 8 * (w.kp->total_warps - vw->active) > w.kp->total_warps;
+      w.h->deep = STM_DEEP_FRAC * (w.kp->total_warps - vw->active) > w.kp->total_warps;
     }
   }
   return __shfl_sync(FULLMASK, want, 0) != 0;
