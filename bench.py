@@ -446,6 +446,7 @@ def main():
         if world > 1:
             dist.barrier()
     got = layer.check(d_res)  # raises if any rank's launch reported a failure status
+    main_info = stm.stm_last_launch()  # the last timed launch (the workload's last query)
     parity = []
     for qi in range(len(plans)):
         if got[qi] != counts[qi]:
@@ -514,7 +515,7 @@ def main():
                           "matches_per_s": counts[qi] / tq if tq else None,
                           "alg_bytes": alg[qi], "merge_bytes": merge[qi], "set_ops": jobs[qi],
                           "idle_steal_fraction": idle[qi], "degree_ranked": ranked[qi]})
-        info = stm.stm_last_launch()
+        info = main_info
         line = {
             "metric": METRIC,
             "value": value, "unit": "matches/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -534,7 +535,8 @@ def main():
                          "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
                          "ncu": ncu_ev,
                          "kernel": ("stm_count_kernel_occ" if info.get("variant") == 2 else "stm_count_kernel")
-                                   + f" ({queries[dom][0]} launch, unroll {info.get('unroll')})",
+                                   + f" ({queries[dom][0]} launch, unroll {info.get('unroll')}, "
+                                   f"{'plan-specialised' if info.get('jit') else 'generic'} kernel)",
                          "algorithmic_bytes_per_launch": alg[dom], "algorithmic_bytes_per_step": W_step,
                          "peak_source": peak_src,
                          "note": "achieved = SURVEY.md 8(d) W of the dominant launch (instrumented launch) / "
